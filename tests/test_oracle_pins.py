@@ -1,0 +1,358 @@
+"""Pins for the CPU oracle (-m "not gpu").  The oracle is trusted only after
+these pass; each check ties it to something other than itself: published
+known answers, closed forms, brute force, an N-version twin, invariants.
+Self-check numbering (i)-(ix) follows SURVEY.md §8c / DESIGN.md §5.
+"""
+import math
+import os
+from collections import defaultdict
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import twin
+from synth import graphs as SG
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+P = (1 << 31) - 1
+
+
+def _gold_lines(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return [ln.split() for ln in f if ln.strip() and not ln.startswith("#")]
+
+
+# ---------------------------------------------------------------- (v) primitives
+def test_splitmix64_known_answers():
+    want = [int(x[0], 16) for x in _gold_lines("splitmix64_seed0.txt")]
+    # the oracle's stream = mix64(state += gamma); with seed 0 the first
+    # three states are gamma, 2 gamma, 3 gamma
+    gamma = 0x9E3779B97F4A7C15
+    got = [oracle.mix64((k * gamma) & ((1 << 64) - 1)) for k in (1, 2, 3)]
+    assert got == want
+
+
+def test_mix64_is_a_bijection_inverse_roundtrip():
+    # closed-form inverse of the splitmix64 finaliser: the two odd multipliers
+    # have inverses 0x96de1b173f119089 and 0x319642b2d24d8ec3 mod 2^64
+    M = (1 << 64) - 1
+
+    def unxs(z, s):
+        x = z
+        for _ in range(64 // s + 1):
+            x = z ^ (x >> s)
+        return x
+
+    def inv(z):
+        z = unxs(z, 31)
+        z = (z * 0x319642B2D24D8EC3) & M
+        z = unxs(z, 27)
+        z = (z * 0x96DE1B173F119089) & M
+        return unxs(z, 30)
+
+    assert (0xBF58476D1CE4E5B9 * 0x96DE1B173F119089) & M == 1
+    assert (0x94D049BB133111EB * 0x319642B2D24D8EC3) & M == 1
+    rng = np.random.default_rng(7)
+    for z in [0, 1, M, 1 << 63] + [int(x) for x in rng.integers(0, 1 << 63, 200, dtype=np.int64)]:
+        assert inv(oracle.mix64(z)) == z
+
+
+def test_hash_adversarial_vectors():
+    for A, B, v, h in (map(int, r) for r in _gold_lines("m31_vectors.txt")):
+        assert oracle.hash1(A, B, v) == h
+        assert (A * v + B) % P == h           # big-int definition
+    # the zero residue in row 1 is the closed form (P - B) * A^(P-2) mod P
+    A, B = 123456789, 987654321
+    assert (P - B) * pow(A, P - 2, P) % P == 773987457
+
+
+def test_hash_random_vs_bigint():
+    rng = np.random.default_rng(11)
+    A = rng.integers(1, P, 20000)
+    B = rng.integers(0, P, 20000)
+    v = rng.integers(0, P, 20000)
+    for a, b, x in zip(A.tolist(), B.tolist(), v.tolist()):
+        assert oracle.hash1(a, b, x) == (a * x + b) % P
+
+
+def test_hash_params_ranges_and_twin():
+    for seed in [0, 1, 101, 2**63 + 5]:
+        A, B = oracle.hash_params(seed, 500)
+        assert A.min() >= 1 and A.max() <= P - 1
+        assert B.max() <= P - 1
+        tA, tB = twin.hash_params(seed, 500)
+        assert A.tolist() == tA and B.tolist() == tB
+
+
+def test_validate_rejects_bad_csr():
+    g = SG.random_graph(50, 200, seed=1)
+    assert oracle.validate(g.row_ptr, g.col)
+    bad = g.col.copy()
+    r = int(np.argmax(np.diff(g.row_ptr) >= 2))
+    a = g.row_ptr[r]
+    bad[a], bad[a + 1] = bad[a + 1], bad[a]          # unsorted row
+    assert not oracle.validate(g.row_ptr, bad)
+    bad = g.col.copy()
+    bad[a + 1] = bad[a]                               # duplicate
+    assert not oracle.validate(g.row_ptr, bad)
+    bad = g.col.copy()
+    bad[-1] = 50                                      # id >= n
+    assert not oracle.validate(g.row_ptr, bad)
+    rp = g.row_ptr.copy()
+    rp[-1] += 1                                       # row_ptr[n] != nnz
+    assert not oracle.validate(rp, g.col)
+
+
+# ---------------------------------------------------------------- (i) top-s == full sort
+@pytest.mark.parametrize("s", [1, 2, 3, 5])
+def test_top_s_equals_bruteforce_full_sort(s):
+    g = SG.make("tiny")
+    c, seed = 12, 99
+    A, B = oracle.hash_params(seed, c)
+    deg = g.degrees()
+    rows = np.nonzero(deg >= s)[0]
+    rng = np.random.default_rng(s)
+    rows = rows[rng.permutation(len(rows))[:800]]
+    for u in rows.tolist():
+        nb = g.col[g.row_ptr[u]:g.row_ptr[u + 1]].astype(np.int64)
+        ids = oracle.row_shingles(nb, s, c, seed, A, B)
+        hv = (A.astype(np.int64)[:, None] * nb[None, :] + B.astype(np.int64)[:, None]) % P
+        hv.sort(axis=1)                                # full sort of every Gamma_j(u)
+        for j in range(c):
+            mins = [int(x) for x in hv[j, :s]]
+            assert int(ids[j]) == twin.shingle_id(s, seed, j, mins)
+
+
+def test_hash_eval_count_matches_complexity():
+    # the work is one hash per (adjacency entry, trial) of every
+    # eligible row in both passes: sum_{deg>=s1} deg*c1 + sum_{S1'} |L|*c2
+    g = SG.make("tiny")
+    s1, c1, s2, c2 = 2, 10, 2, 7
+    res = oracle.shingling(g.row_ptr, g.col, s1, c1, 3, s2, c2, 4)
+    d = g.degrees()
+    want1 = int(d[d >= s1].sum()) * c1
+    sizes = np.diff(res.G1.offs)
+    want2 = int(sizes[sizes >= s2].sum()) * c2
+    assert res.hash_evals == want1 + want2
+
+
+# ---------------------------------------------------------------- (ii) twins
+def test_identical_neighbourhoods_identical_shingles():
+    rng = np.random.default_rng(3)
+    n = 400
+    adj = [set() for _ in range(n)]
+    for _ in range(3000):
+        a, b = rng.integers(0, n, 2)
+        if a != b:
+            adj[a].add(int(b)); adj[b].add(int(a))
+    # make 300 and 301 twins: same neighbourhood, not adjacent to each other
+    adj[300].discard(301); adj[301].discard(300)
+    for v in list(adj[301]):
+        adj[v].discard(301)
+    for v in adj[300]:
+        adj[v].add(301)
+    adj[301] = set(adj[300])
+    g = SG.from_adj([sorted(x) for x in adj])
+    res = oracle.shingling(g.row_ptr, g.col, 2, 64, 5, 2, 16, 6)
+    r = {int(u): i for i, u in enumerate(res.rows1)}
+    assert np.array_equal(res.M1[r[300]], res.M1[r[301]])
+    # and both are members of exactly the same first-level groups
+    for j in range(64):
+        lo, hi = res.G1.trial_goffs[j], res.G1.trial_goffs[j + 1]
+        for gi in range(lo, hi):
+            mem = res.G1.members[res.G1.offs[gi]:res.G1.offs[gi + 1]]
+            assert (300 in mem) == (301 in mem)
+
+
+# ---------------------------------------------------------------- (iii) planted cliques
+@pytest.mark.parametrize("mode", [0, 1])
+def test_planted_cliques_one_cluster_each(mode):
+    sizes = [5, 6, 8, 10, 12, 15, 20, 25, 30, 9, 7, 11]
+    g = SG.cliques(sizes, n=sum(sizes) + 40, seed=17)     # + 40 isolated vertices
+    res = oracle.shingling(g.row_ptr, g.col, 2, 100, 21, 2, 100, 22)
+    labels, nc = res.report(mode=mode)
+    assert nc == len(sizes)
+    # each clique is one CC of G: compare the label partition with the CCs
+    deg = g.degrees()
+    comp = _components(g)
+    for v in range(g.n):
+        if deg[v] == 0:
+            assert labels[v] == v
+    by_label = defaultdict(set)
+    by_comp = defaultdict(set)
+    for v in range(g.n):
+        by_label[labels[v]].add(v)
+        by_comp[comp[v]].add(v)
+    assert sorted(map(sorted, by_label.values())) == sorted(map(sorted, by_comp.values()))
+
+
+def _components(g):
+    n = g.n
+    lab = -np.ones(n, np.int64)
+    for s in range(n):
+        if lab[s] >= 0:
+            continue
+        lab[s] = s
+        st = [s]
+        while st:
+            x = st.pop()
+            for y in g.col[g.row_ptr[x]:g.row_ptr[x + 1]]:
+                if lab[y] < 0:
+                    lab[y] = s
+                    st.append(int(y))
+    return lab
+
+
+# ---------------------------------------------------------------- (iv) min-wise rate
+def _binom_two_sided_tail(k, n, p):
+    """Exact two-sided binomial tail probability P(|X - np| >= |k - np|)."""
+    mean = n * p
+    d = abs(k - mean)
+    logs = [math.lgamma(n + 1) - math.lgamma(i + 1) - math.lgamma(n - i + 1)
+            + (i * math.log(p) if i else 0.0) + ((n - i) * math.log1p(-p) if n - i else 0.0)
+            for i in range(n + 1)]
+    return min(1.0, sum(math.exp(l) for i, l in enumerate(logs) if abs(i - mean) >= d - 1e-9))
+
+
+@pytest.mark.parametrize("s,inter,union", [(1, 10, 40), (2, 30, 60), (2, 12, 30), (3, 40, 60)])
+def test_minwise_collision_rate_matches_closed_form(s, inter, union):
+    # [4] via P:L437-439: Pr[top-s(A) = top-s(B)] = C(|A n B|, s) / C(|A u B|, s)
+    # (= Jaccard, Eq. 1, for s = 1).  Ids must be scattered.
+    rng = np.random.default_rng(1000 + s * 100 + inter)
+    ids = rng.choice(1_000_000, union, replace=False).astype(np.uint32)
+    half = (union - inter) // 2
+    Aset = np.sort(ids[: inter + half])
+    Bset = np.sort(np.concatenate([ids[:inter], ids[inter + half:]]))
+    T = 10_000
+    sa = oracle.row_shingles(Aset, s, T, 4242)
+    sb = oracle.row_shingles(Bset, s, T, 4242)
+    hits = int((sa == sb).sum())
+    p = math.comb(inter, s) / math.comb(len(np.union1d(Aset, Bset)), s)
+    assert T * p >= 20
+    assert _binom_two_sided_tail(hits, T, p) >= 1e-6, (hits, T * p)
+
+
+# ---------------------------------------------------------------- (vi) ids and grouping
+def test_s_le_2_ids_roundtrip_through_A_inverse():
+    g = SG.make("tiny")
+    for s in (1, 2):
+        res = oracle.shingling(g.row_ptr, g.col, s, 8, 31, 2, 4, 32)
+        for r in range(0, len(res.rows1), 97):
+            u = int(res.rows1[r])
+            nb = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
+            for j in range(8):
+                idv = int(res.M1[r, j])
+                hs = [idv] if s == 1 else [idv >> 31, idv & P]
+                A, B = int(res.A1[j]), int(res.B1[j])
+                Ainv = pow(A, P - 2, P)
+                verts = sorted((h - B) * Ainv % P for h in hs)
+                want = sorted(oracle.row_constituents(nb, s, A, B).tolist())
+                assert verts == want
+                assert all(v in set(nb.tolist()) for v in verts)
+
+
+def test_exact_tuple_grouping_equals_id_grouping_s3():
+    g = SG.make("tiny")
+    s, c, seed = 3, 10, 77
+    res = oracle.shingling(g.row_ptr, g.col, s, c, seed, 2, 3, 78)
+    A, B = res.A1, res.B1
+    for j in range(c):
+        tup = defaultdict(list)
+        for r, u in enumerate(res.rows1.tolist()):
+            nb = g.col[g.row_ptr[u]:g.row_ptr[u + 1]].astype(np.int64)
+            hv = np.sort((int(A[j]) * nb + int(B[j])) % P)[:s]
+            tup[tuple(hv.tolist())].append(u)
+        lo, hi = res.G1.trial_goffs[j], res.G1.trial_goffs[j + 1]
+        groups = sorted(res.G1.members[res.G1.offs[k]:res.G1.offs[k + 1]].tolist() for k in range(lo, hi))
+        assert groups == sorted(sorted(v) for v in tup.values())
+
+
+def test_group_invariants():
+    g = SG.make("tiny")
+    res = oracle.shingling(g.row_ptr, g.col, 2, 20, 1, 2, 20, 2)
+    for G, nrows, c in ((res.G1, len(res.rows1), 20), (res.G2, len(res.s1p_group), 20)):
+        assert G.offs[-1] == nrows * c                # sum |L| = rows * c
+        for j in range(c):
+            lo, hi = G.trial_goffs[j], G.trial_goffs[j + 1]
+            keys = [oracle.mix64(int(x)) for x in G.ids[lo:hi]]
+            assert keys == sorted(keys) and len(set(keys)) == len(keys)
+            assert G.offs[hi] - G.offs[lo] == nrows
+        for k in range(len(G.ids)):
+            m = G.members[G.offs[k]:G.offs[k + 1]]
+            assert len(m) >= 1 and np.all(np.diff(m.astype(np.int64)) > 0)
+
+
+# ---------------------------------------------------------------- (vii) CC-locality
+def test_cc_locality():
+    g = SG.make("tiny")
+    comp = _components(g)
+    roots = np.unique(comp[g.degrees() > 0])
+    part = np.isin(comp, roots[::2])            # half of the components
+    runs = []
+    for keep in (part, ~part):
+        rp = np.zeros(g.n + 1, np.int64)
+        d = np.where(keep, g.degrees(), 0)
+        rp[1:] = np.cumsum(d)
+        col = np.concatenate([g.col[g.row_ptr[u]:g.row_ptr[u + 1]] for u in range(g.n) if keep[u]])
+        runs.append(oracle.shingling(rp, col, 2, 30, 9, 2, 30, 10))
+    full = oracle.shingling(g.row_ptr, g.col, 2, 30, 9, 2, 30, 10)
+    # pass-1 shingles of each vertex depend only on its own component
+    rowmap = {int(u): i for i, u in enumerate(full.rows1)}
+    for r in runs:
+        for i, u in enumerate(r.rows1.tolist()):
+            assert np.array_equal(r.M1[i], full.M1[rowmap[u]])
+    # first-level groups of the union = union of the parts' groups (per trial)
+    for j in range(30):
+        def gs(res):
+            lo, hi = res.G1.trial_goffs[j], res.G1.trial_goffs[j + 1]
+            return {(int(res.G1.ids[k]), tuple(res.G1.members[res.G1.offs[k]:res.G1.offs[k + 1]].tolist()))
+                    for k in range(lo, hi)}
+        assert gs(full) == gs(runs[0]) | gs(runs[1])
+    # final clusters of the union = union of the parts' clusters
+    lf, _ = full.report()
+    for r, keep in zip(runs, (part, ~part)):
+        lr, _ = r.report()
+        assert np.array_equal(lf[keep], lr[keep])
+
+
+# ---------------------------------------------------------------- (viii)+(ix) N-version
+@pytest.mark.parametrize("s1,c1,s2,c2,gseed", [(2, 6, 2, 5, 1), (1, 5, 1, 4, 2), (3, 6, 2, 4, 3),
+                                             (2, 9, 3, 5, 4), (5, 4, 2, 6, 5)])
+def test_oracle_equals_python_twin(s1, c1, s2, c2, gseed):
+    # a small graph with dense pockets so that groups of size >= s2 exist
+    g = SG.homology_graph(n=300, n_isolated=20, m_target=2500, seed=gseed, n_cliques=3,
+                          clique_lo=6, clique_hi=12, cc_max=120, fam_hi=40)
+    g = SG.Graph(*g)
+    res = oracle.shingling(g.row_ptr, g.col, s1, c1, 100 + gseed, s2, c2, 200 + gseed)
+    tw = twin.shingling(SG.to_adj(g), s1, c1, 100 + gseed, s2, c2, 200 + gseed)
+    assert res.rows1.tolist() == tw["rows1"]
+    assert res.M1.tolist() == tw["M1"]
+
+    def flat(G, c):
+        out = []
+        for j in range(c):
+            for k in range(G.trial_goffs[j], G.trial_goffs[j + 1]):
+                out.append((j, int(G.ids[k]), G.members[G.offs[k]:G.offs[k + 1]].tolist()))
+        return out
+
+    assert flat(res.G1, c1) == tw["G1"]
+    assert res.s1p_group.tolist() == tw["s1p"]
+    assert res.M2.tolist() == tw["M2"]
+    assert flat(res.G2, c2) == tw["G2"]
+    for mode in (0, 1):
+        for ms in (1, 3):
+            lab, nc = res.report(mode=mode, min_size=ms)
+            tl, tn = twin.report(tw, mode=mode, min_size=ms)
+            assert lab.tolist() == tl and nc == tn
+
+
+def test_report_labels_are_min_of_class():
+    g = SG.make("tiny")
+    res = oracle.shingling(g.row_ptr, g.col, 2, 30, 1, 2, 30, 2)
+    lab, nc = res.report()
+    classes = defaultdict(list)
+    for v, l in enumerate(lab.tolist()):
+        classes[l].append(v)
+    assert all(min(vs) == l for l, vs in classes.items())
+    assert nc == sum(1 for vs in classes.values() if len(vs) >= 2)
