@@ -1,0 +1,365 @@
+#!/usr/bin/env python3
+"""Benchmark: edges/sec shingled (2 passes, device-timed, max over ranks).
+
+One step = one pass of the whole hot path: pass I min-hash top-s
+-> group I -> pass II -> group II, on the synthetic GOS-shaped 2M-vertex graph
+(BASELINE.json configs[1]; s1 = s2 = 2, c1 = c2 = 200) with the CSR already
+resident in HBM.  Prints ONE JSON line (rank 0).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+--impl reference times the CPU oracle (oracle/, the plain single-threaded C
+program written from the paper) on a bounded row sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import platform
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import graphs as SG  # noqa: E402
+
+METRIC = "edges/sec shingled (2 passes, device-timed, max over ranks)"
+UNIT = "edges/s"
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return dict(hbm=d.get("hbm_gbs", 6650.0), sm_max_mhz=d.get("sm_max_mhz", 1965.0),
+                    src="measured (MEASURED_PEAKS.json)")
+    return dict(hbm=6650.0, sm_max_mhz=1965.0, src="fallback (B200_PROFILING.md)")
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev: int):
+        self.dev = dev
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100", "-i", str(self.dev)],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+            time.sleep(0.25)
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": mx, "reasons": [], "samples": 0}
+        busy = [x for x in sm if x > 0.5 * (mx or 1965)] or sm
+        return {"sm_mhz": float(np.median(busy)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- workload
+def workload(name: str):
+    cfg = SG.CONFIGS[name]
+    g = SG.make(name, cache=os.environ.get("SG_BENCH_CACHE", "0") == "1")
+    return g, cfg
+
+
+def oracle_sample(g, target_nnz: int):
+    """Row-prefix sample: rows [0, u) keep their full adjacency lists, later
+    rows are emptied (a valid CSR: the oracle accepts asymmetric rows)."""
+    u = int(np.searchsorted(g.row_ptr, target_nnz))
+    u = max(1, min(u, g.n))
+    rp = g.row_ptr.copy()
+    rp[u + 1:] = rp[u]
+    col = np.ascontiguousarray(g.col[:rp[u]])
+    return rp, col, u
+
+
+def run_oracle(g, cfg, target_nnz):
+    import oracle
+    rp, col, u = oracle_sample(g, target_nnz)
+    t0 = time.perf_counter()
+    oracle.shingling(rp, col, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    dt = time.perf_counter() - t0
+    edges = len(col) / 2.0
+    return edges / dt, dt, u, len(col)
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return platform.processor()
+
+
+# ---------------------------------------------------------------- roofline
+def roofline_table(stage_ms: dict, counts: dict, work: dict, pk: dict):
+    """Per-kernel algorithmic work / device time."""
+    hbm = pk["hbm"]
+    issue_peak = 148 * 128 * pk["sm_max_mhz"] * 1e6 / 1e12     # T thread-instr/s
+    P1, P2 = counts["pairs1"], counts["pairs2"]
+    rows = {}
+
+    def hbm_row(stage, nbytes):
+        t = stage_ms.get(stage, 0.0) / 1e3
+        if t <= 0:
+            return None
+        a = nbytes / t / 1e9
+        return {"bound": "hbm", "achieved": round(a, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(a / hbm, 4), "ms": round(stage_ms[stage], 3), "bytes": int(nbytes)}
+
+    def alu_row(stage, entry_trials):
+        t = stage_ms.get(stage, 0.0) / 1e3
+        if t <= 0:
+            return None
+        a = 7.0 * entry_trials / t / 1e12                      # 7 algorithmic instr / (entry, trial)
+        return {"bound": "alu", "achieved": round(a, 3), "peak": round(issue_peak, 2),
+                "unit": "T instr/s", "frac": round(a / issue_peak, 4), "ms": round(stage_ms[stage], 3),
+                "entry_trials": int(entry_trials)}
+
+    rows["hash1"] = alu_row("hash1", work["et1"])
+    rows["hash2"] = alu_row("hash2", work["et2"])
+    for lv, P in ((1, P1), (2, P2)):
+        # hist+offsets: read 8 B key/pair; scatter: read 8 B key + write 12 B pair;
+        # local: read 12 B pair + write 4 B member + 1 head bit per pair
+        rows[f"hist{lv}"] = hbm_row(f"hist{lv}", 8 * P)
+        rows[f"scatter{lv}"] = hbm_row(f"scatter{lv}", 20 * P)
+        rows[f"local{lv}"] = hbm_row(f"local{lv}", 16.125 * P)
+    return {k: v for k, v in rows.items() if v}
+
+
+# ---------------------------------------------------------------- our arm
+def bench_ours(args, rank, world, local_rank):
+    import torch
+    from paper_conf_ipps_wuk13_b200 import binding as B
+    torch.cuda.set_device(local_rank)
+    dist_on = world > 1
+    if dist_on:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    g, cfg = workload(args.config)
+    s1, c1, seed1, s2, c2, seed2 = (cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    stream = torch.cuda.current_stream()
+    dinfo = {"rank": rank, "world": world, "device": local_rank, "stream": stream.cuda_stream}
+    if dist_on:
+        uid = [None]
+        if rank == 0:
+            uid[0] = B.nccl_unique_id()
+        torch.distributed.broadcast_object_list(uid, src=0)
+        dinfo["nccl_uid"] = uid[0]
+    # pinned host copy of the input (used by the e2e leg)
+    rp_pin = torch.from_numpy(g.row_ptr).pin_memory()
+    col_pin = torch.from_numpy(g.col).pin_memory()
+    h = B.shingle_graph_create(rp_pin.numpy(), col_pin.numpy(), dist=dinfo)
+
+    def step():
+        B.shingle_graph_reset(h)
+        B.shingle_pass(h, s1, c1, seed1)
+        B.group_by_shingle(h)
+        B.shingle_pass(h, s2, c2, seed2)
+        B.group_by_shingle(h)
+
+    def barrier():
+        if dist_on:
+            torch.distributed.barrier()
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    stage_sum = {}
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+            for k, v in B.sg_get_stage_ms(h).items():
+                stage_sum[k] = stage_sum.get(k, 0.0) + v
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    if dist_on:
+        t = torch.tensor([ms], device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    counts = B.sg_get_counts(h)
+    stage_ms = {k: v / args.steps for k, v in stage_sum.items()}
+    # algorithmic work of the two min-hash passes: entry x trial
+    deg = g.degrees()
+    et1 = float(deg[deg >= s1].sum()) * c1
+    et2 = float(counts["entries2"]) * c2      # pass-II entries = sum |L| over S1'
+    launches = counts["launches"]              # kernels of the last step (counter reset each step)
+    B.shingle_graph_destroy(h)
+
+    # ---- e2e: the public API with host buffers, H2D + D2H inside the region
+    e2e = None
+    if not args.no_e2e:
+        torch.cuda.synchronize()
+        barrier()
+        t0 = time.perf_counter()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            hh = B.shingle_graph_create(rp_pin.numpy(), col_pin.numpy(), dist=dinfo)
+            B.shingle_pass(hh, s1, c1, seed1)
+            B.group_by_shingle(hh)
+            B.shingle_pass(hh, s2, c2, seed2)
+            B.group_by_shingle(hh)
+            res = B.sg_get_counts(hh)      # D2H of the step's result summary
+            B.shingle_graph_destroy(hh)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        wall = (time.perf_counter() - t0) / args.steps * 1e3
+        ems = max(e0.elapsed_time(e1) / args.steps, wall)
+        if dist_on:
+            t = torch.tensor([ems], device="cuda")
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": round(g.m / (ems / 1e3), 1), "unit": UNIT,
+               "h2d_bytes_per_step": int(g.row_ptr.nbytes + g.col.nbytes) // max(world, 1),
+               "d2h_bytes_per_step": 80, "ms_per_step": round(ems, 3),
+               "includes": "create (H2D from pinned host + device CSR validation) + 2 passes + 2 groupings + counts D2H + destroy"}
+
+    if rank != 0:
+        if dist_on:
+            torch.distributed.destroy_process_group()
+        return
+    work = {"et1": et1, "et2": et2}
+    pk = peaks()
+    rt = roofline_table(stage_ms, counts, work, pk)
+    dom_name = max(rt, key=lambda k: rt[k]["ms"]) if rt else None
+    dom = dict(rt[dom_name]) if dom_name else None
+    if dom:
+        dom["kernel"] = dom_name
+        dom["traffic"] = None
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        v, dt, u, nnz_s = run_oracle(g, cfg, args.cpu_sample_nnz)
+        cpu = {"value": round(v, 1), "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"row prefix of the same graph: rows [0,{u}) with full adjacency ({nnz_s} entries, "
+                         f"{nnz_s // 2} edges), full two-pass method, {dt:.1f} s single-threaded",
+               "host_cpu": cpu_model(), "host_cores": os.cpu_count()}
+    clocks = clk.summary()
+    out = {
+        "metric": METRIC, "value": round(g.m * world / world / (ms / 1e3), 1), "unit": UNIT,
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u32/u64 (integer)", "data": "synthetic (seeded homology-like generator, synth/graphs.py)",
+        "config": {"workload": f"{args.config}: n={g.n} m={g.m} (nnz={g.nnz}), s1={s1} c1={c1} s2={s2} c2={c2}",
+                   "n_e": counts["n_e"], "groups1": counts["groups1"], "s1p": counts["s1p"],
+                   "groups2": counts["groups2"], "pairs1": counts["pairs1"], "pairs2": counts["pairs2"],
+                   "l2": "inputs larger than L2 (CSR %.0f MB; per-step intermediates several GB)" % ((g.row_ptr.nbytes + g.col.nbytes) / 1e6),
+                   "parallelism": f"vertex-range shards x{world}"},
+        "stage_ms": {k: round(v, 3) for k, v in stage_ms.items() if v > 0},
+        "roofline": dom, "roofline_stages": rt, "peak_source": pk["src"],
+        "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches * args.steps,
+        "gpu_launches_per_step": launches,
+        "clocks": clocks,
+    }
+    print(json.dumps(out))
+    if dist_on:
+        torch.distributed.destroy_process_group()
+
+
+# ---------------------------------------------------------------- reference arm
+def bench_reference(args, rank, world):
+    if rank != 0:
+        return
+    g, cfg = workload(args.config)
+    vals, dts = [], []
+    for i in range(args.warmup + args.steps):
+        v, dt, u, nnz_s = run_oracle(g, cfg, args.ref_sample_nnz)
+        if i >= args.warmup:
+            vals.append(v)
+            dts.append(dt)
+    v = float(np.median(vals))
+    out = {"metric": METRIC, "value": round(v, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(float(np.median(dts)) * 1e3, 1),
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+           "dtype": "u32/u64 (integer)", "data": "synthetic (seeded homology-like generator)",
+           "config": {"workload": f"{args.config} (row-prefix sample: {nnz_s} of {g.nnz} entries)"},
+           "impl": "reference",
+           "cpu_baseline": {"value": round(v, 1), "unit": UNIT, "cores": 1, "kind": "oracle",
+                            "sample": f"rows [0,{u}) of {args.config} with full adjacency ({nnz_s} entries)",
+                            "host_cpu": cpu_model(), "host_cores": os.cpu_count()},
+           "e2e": {"value": round(v, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="gos2m")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample-nnz", type=int, default=1_500_000)
+    ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        bench_reference(args, rank, world)
+    else:
+        bench_ours(args, rank, world, local_rank)
+
+
+if __name__ == "__main__":
+    main()

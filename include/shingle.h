@@ -1,0 +1,195 @@
+/*
+ * shingle.h — C ABI of libshingle.so, the B200 (sm_100a) implementation of the
+ * data-parallel hot path of Wu & Kalyanaraman's GPU Shingling (gpClust,
+ * IPDPSW 2013): the two-pass min-wise shingle generation of Gibson et al.
+ *
+ * Citations "P:Lx-y" are lines of the paper text (reference PAPER.md);
+ * "AMB-n" are the readings of silent/garbled passages fixed in DESIGN.md §3.
+ *
+ * Conventions for every call:
+ *  - plain C types only; no exceptions cross the ABI; every call returns an
+ *    sg_status (or void for destroy);
+ *  - host pointers are borrowed for the duration of the call only; device
+ *    memory is owned by the handle and released by shingle_graph_destroy;
+ *  - all device work is enqueued on the handle's stream (sg_dist.stream, or a
+ *    stream the library creates); each call returns when its stage has
+ *    completed on the device (it synchronises the stream);
+ *  - after SG_ECUDA or SG_ENCCL the handle is poisoned: every later call
+ *    except destroy / sg_last_error returns the same status;
+ *  - the library never falls back to a CPU implementation: without a usable
+ *    CUDA device shingle_graph_create returns SG_ECUDA.
+ */
+#ifndef SHINGLE_H
+#define SHINGLE_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SG_API __attribute__((visibility("default")))
+#else
+#define SG_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum sg_status {
+    SG_OK = 0,
+    SG_EINVAL = 1,     /* invalid argument or invalid CSR (see create) */
+    SG_ENOMEM = 2,     /* device allocation failed (sg_last_error names the bytes) */
+    SG_ESTATE = 3,     /* call out of order (see the state machine below) */
+    SG_ECUDA = 4,      /* CUDA error / no device; the handle is poisoned */
+    SG_ENCCL = 5,      /* NCCL error in a multi-GPU exchange; handle poisoned */
+    SG_EOVERFLOW = 6   /* a count exceeds 2^32 - 1 (members / rows are u32) */
+} sg_status;
+
+typedef struct sg_graph sg_graph;
+
+/* create() flags */
+#define SG_DEVICE_PTRS 0x1u   /* row_ptr / col are device pointers (on dist->device) */
+#define SG_NO_VALIDATE 0x2u   /* skip the CSR validation (caller guarantees it)   */
+
+/* Multi-GPU description: one process (or, with loopback, one host thread) per
+ * rank, vertex-range sharding, owner-routed exchange before each grouping
+ * (DESIGN.md §7).  NULL = one GPU, current device, library-created stream. */
+typedef struct sg_dist {
+    int32_t rank;              /* 0 <= rank < world */
+    int32_t world;             /* number of ranks (>= 1) */
+    int32_t device;            /* CUDA device ordinal used by this rank */
+    void *stream;              /* cudaStream_t to enqueue on, or NULL */
+    const uint8_t *nccl_uid;   /* 128-byte ncclUniqueId (world > 1, NCCL backend) */
+    void *loopback;            /* sg_loopback* (world > 1, in-process test backend) or NULL */
+} sg_dist;
+
+/* ------------------------------------------------------------------------ */
+/* shingle_graph_create — ingest an unweighted G(V, E) given as adjacency   */
+/* lists ("the graph is made available as an adjacency list";   */
+/* one contiguous array + boundary marks = CSR).                */
+/*   n        number of vertices; 0 <= n < P = 2^31 - 1 (AMB-1: ids must be */
+/*            < P for (A*v + B) % P to be a bijection)          */
+/*   nnz      number of adjacency entries (2m for an undirected graph)      */
+/*   row_ptr  int64[n+1], row_ptr[0] = 0, row_ptr[n] = nnz, non-decreasing  */
+/*   col      int32[nnz], each row strictly increasing, 0 <= col < n         */
+/*            (AMB-8: duplicates rejected; self-loops/asymmetry accepted)   */
+/*   flags    SG_DEVICE_PTRS, SG_NO_VALIDATE                                */
+/*   dist     NULL or the rank description above                           */
+/*   out      receives the handle (NULL on failure)                         */
+/* The whole CSR is global; each rank copies its own row range into HBM.   */
+/* Errors: SG_EINVAL (bad arguments / CSR), SG_ENOMEM, SG_ECUDA, SG_ENCCL.  */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr,
+                               const int32_t *col, uint32_t flags, const sg_dist *dist,
+                               sg_graph **out);
+
+/* ------------------------------------------------------------------------ */
+/* shingle_pass — one shingling pass (Alg. 1).      */
+/* First call: Pass I over G.  Second call (after group_by_shingle): Pass II */
+/* over G_I, whose rows are the member lists L(s) of the first-level         */
+/* shingles with |L| >= s (S1', AMB-6).                          */
+/* For every row with at least s entries and every trial       */
+/* j < c: the s smallest h_j(v) = (A_j v + B_j) mod P over the row (AMB-7),  */
+/* folded into a within-trial shingle id (AMB-4: s=1: h1; s=2:               */
+/* h1*2^31 + h2; s>=3: 64-bit splitmix fold).  (A_j, B_j) come from a        */
+/* splitmix64 stream seeded with `seed` (AMB-2).                            */
+/*   s in [1, 8] (s "typically under 10"), c in [1, 1024].       */
+/* Errors: SG_EINVAL (s, c), SG_ESTATE (wrong order), SG_ENOMEM, SG_ECUDA,  */
+/* SG_EOVERFLOW (rows * c >= 2^32 on one rank).                              */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed);
+
+/* ------------------------------------------------------------------------ */
+/* group_by_shingle — "a sorting is done to gather all vertices that         */
+/* generated each shingle ... once for each random trial" (P:L404-410,       */
+/* AMB-5): per trial, the <shingle, generator> pairs of the last pass are    */
+/* grouped into tuples <s_j, L(s_j)>, giving G_I after pass I   */
+/* and G_II after pass II.  Canonical order (AMB-19): trials    */
+/* ascending; within a trial, groups by key = splitmix64-finaliser(id)       */
+/* ascending; members ascending.  With world > 1 the pairs are first routed */
+/* to the rank owning their key (NCCL all-to-all).                           */
+/* Errors: SG_ESTATE, SG_ENOMEM, SG_ECUDA, SG_ENCCL, SG_EOVERFLOW.           */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status group_by_shingle(sg_graph *g);
+
+/* ------------------------------------------------------------------------ */
+/* report_dense_subgraphs — Phase III, approach 2: */
+/* union-find of size n; for each connected component of G_II, union the    */
+/* vertices of G that constitute its first- and second-level shingles       */
+/* (mode 0, AMB-9) or that generated its first-level shingles (mode 1).     */
+/*   labels     host int32[n], caller-allocated; labels[v] = smallest vertex */
+/*              of v's cluster (AMB-10); clusters smaller than min_size are  */
+/*              reported as singletons (labels[v] = v).  Filled on rank 0;   */
+/*              other ranks may pass NULL.                                   */
+/*   n_clusters receives the number of clusters with >= max(2, min_size)     */
+/*              vertices (may be NULL).                                      */
+/* Host work, outside the timed hot path.  Requires state GROUPED2.          */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
+                                 int64_t *n_clusters);
+
+/* Return the handle to state CREATED (CSR kept, results dropped) so the two */
+/* passes can be run again, e.g. by a benchmark.                             */
+SG_API sg_status shingle_graph_reset(sg_graph *g);
+
+SG_API void shingle_graph_destroy(sg_graph *g);
+
+/* Last error message of the handle (or of the calling thread if g == NULL). */
+SG_API const char *sg_last_error(const sg_graph *g);
+
+/* ------------------------------------------------------------------------ */
+/* Getters (host buffers; two-call pattern: NULL buffers report sizes).      */
+/* ------------------------------------------------------------------------ */
+
+/* counts[0..11] = n, this rank's first row, rows on this rank, n_e (pass-I  */
+/* rows, global), |S1| (G_I groups), |S1'| (pass-II rows), |S2| (G_II        */
+/* groups), P1 pairs, P2 pairs, state, E2 (pass-II entries = sum of |L| over */
+/* S1'), device-kernel launches since create / the last reset.  Global      */
+/* counts are summed over ranks.                                             */
+SG_API sg_status sg_get_counts(const sg_graph *g, int64_t counts[12]);
+
+/* Shingle matrix of pass `level` (1 or 2) on this rank: ids[rows x c]      */
+/* row-major (rows ascending: pass I = vertices with deg >= s1 ascending;   */
+/* pass II = S1' indices ascending), plus the row's generator value in       */
+/* rowid[rows] (pass I: vertex id; pass II: S1' index).                      */
+SG_API sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *rowid,
+                          int64_t cap_rows, int64_t *rows, int32_t *c);
+
+/* Groups of level 1 (G_I) or 2 (G_II) owned by this rank, canonical order:  */
+/*   trial_goffs[c+1] group ranges per trial, ids[G], offs[G+1] (into        */
+/*   members), members[Pairs].  caps = {G, Pairs}; counts <- {G, Pairs, c}.  */
+SG_API sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64_t *ids,
+                        int64_t *offs, uint32_t *members, const int64_t caps[2],
+                        int64_t counts[3]);
+
+/* The S1' map: s1p_group[k] = index (in this rank's G_I, canonical order)   */
+/* of first-level shingle k; first global index of this rank in *k0.        */
+SG_API sg_status sg_get_s1p(sg_graph *g, int64_t *s1p_group, int64_t cap, int64_t *count, int64_t *k0);
+
+/* Hash pairs of pass `level`: A[c], B[c]. */
+SG_API sg_status sg_get_hash_params(sg_graph *g, int32_t level, uint32_t *A, uint32_t *B, int32_t cap);
+
+/* Device milliseconds of the last stages (CUDA events on the handle's      */
+/* stream): [0] pass I, [1] group I, [2] pass II, [3] group II, then         */
+/* sub-stage detail.  *n receives the number written.     */
+SG_API sg_status sg_get_stage_ms(const sg_graph *g, float *ms, int32_t cap, int32_t *n);
+
+/* Multi-GPU in-process test backend: `world` virtual ranks on one device,   */
+/* each driven by its own host thread, exchanging through device memcpy.     */
+typedef struct sg_loopback sg_loopback;
+SG_API sg_status sg_loopback_create(int32_t world, sg_loopback **out);
+SG_API void sg_loopback_destroy(sg_loopback *lb);
+
+/* Host-side vertex-range partition used by create: splits   */
+/* [0, n) into `world` contiguous ranges balancing sum(deg + kappa).  bounds */
+/* receives world + 1 row indices.  Pure host code (testable without GPU).   */
+SG_API sg_status sg_partition_rows(int64_t n, const int64_t *row_ptr, int32_t world, int64_t kappa,
+                            int64_t *bounds);
+
+/* Library version / build string (sm_100a). */
+SG_API const char *sg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SHINGLE_H */

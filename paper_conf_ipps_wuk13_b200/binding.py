@@ -1,0 +1,258 @@
+"""ctypes binding of libshingle.so (include/shingle.h) — argument marshalling only.
+
+Every step of the hot path runs in the library's CUDA kernels; this module
+never computes any part of the method and has no CPU fallback: if the shared
+library or a CUDA device is missing, the calls raise.
+Function names mirror the C ABI one to one.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libshingle.so")
+
+SG_OK, SG_EINVAL, SG_ENOMEM, SG_ESTATE, SG_ECUDA, SG_ENCCL, SG_EOVERFLOW = range(7)
+SG_DEVICE_PTRS = 0x1
+SG_NO_VALIDATE = 0x2
+STATUS_NAMES = {0: "SG_OK", 1: "SG_EINVAL", 2: "SG_ENOMEM", 3: "SG_ESTATE", 4: "SG_ECUDA",
+                5: "SG_ENCCL", 6: "SG_EOVERFLOW"}
+STAGES = ["pass1", "group1", "pass2", "group2", "select1", "hash1", "select2", "hash2",
+          "hist1", "scatter1", "local1", "hist2", "scatter2", "local2", "exchange1", "exchange2"]
+
+
+class SGError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS_NAMES.get(status, status)}: {msg}")
+        self.status = status
+
+
+class sg_dist(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("device", C.c_int32),
+                ("stream", C.c_void_p), ("nccl_uid", C.c_void_p), ("loopback", C.c_void_p)]
+
+
+_lib = None
+
+
+def lib() -> C.CDLL:
+    """Load libshingle.so (built by __graft_entry__.build()).  Raises if absent."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = C.CDLL(LIB_PATH)
+    i32, i64, u32, u64, vp = C.c_int32, C.c_int64, C.c_uint32, C.c_uint64, C.c_void_p
+    st = C.c_int
+    sig = {
+        "shingle_graph_create": (st, [i64, i64, vp, vp, u32, vp, C.POINTER(vp)]),
+        "shingle_pass": (st, [vp, i32, i32, u64]),
+        "group_by_shingle": (st, [vp]),
+        "report_dense_subgraphs": (st, [vp, i32, i32, vp, vp]),
+        "shingle_graph_reset": (st, [vp]),
+        "shingle_graph_destroy": (None, [vp]),
+        "sg_last_error": (C.c_char_p, [vp]),
+        "sg_get_counts": (st, [vp, vp]),
+        "sg_get_shingles": (st, [vp, i32, vp, vp, i64, vp, vp]),
+        "sg_get_groups": (st, [vp, i32, vp, vp, vp, vp, vp, vp]),
+        "sg_get_s1p": (st, [vp, vp, i64, vp, vp]),
+        "sg_get_hash_params": (st, [vp, i32, vp, vp, i32]),
+        "sg_get_stage_ms": (st, [vp, vp, i32, vp]),
+        "sg_loopback_create": (st, [i32, C.POINTER(vp)]),
+        "sg_loopback_destroy": (None, [vp]),
+        "sg_partition_rows": (st, [i64, vp, i32, i64, vp]),
+        "sg_version": (C.c_char_p, []),
+    }
+    for name, (rt, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = rt
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+def _check(rc: int, h=None):
+    if rc != SG_OK:
+        msg = lib().sg_last_error(h)
+        raise SGError(rc, msg.decode() if msg else "")
+
+
+def _addr(x) -> int:
+    """Data address of a numpy array or a torch tensor."""
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return x.data_ptr()
+
+
+def _is_cuda(x) -> bool:
+    return hasattr(x, "is_cuda") and x.is_cuda
+
+
+# ------------------------------------------------------------------ C ABI calls
+def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dict] = None):
+    """row_ptr int64[n+1], col int32[nnz]: numpy arrays (host) or CUDA tensors."""
+    dev = _is_cuda(row_ptr)
+    if not dev:
+        row_ptr = np.ascontiguousarray(row_ptr, np.int64)
+        col = np.ascontiguousarray(col, np.int32)
+    n = int(row_ptr.shape[0]) - 1
+    nnz = int(col.shape[0])
+    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE)
+    dptr = None
+    if dist is not None:
+        d = sg_dist(int(dist.get("rank", 0)), int(dist.get("world", 1)), int(dist.get("device", 0)),
+                    dist.get("stream"), None, dist.get("loopback"))
+        uid = dist.get("nccl_uid")
+        if uid is not None:
+            d._uid_buf = C.create_string_buffer(bytes(uid), 128)
+            d.nccl_uid = C.cast(d._uid_buf, C.c_void_p)
+        dptr = C.byref(d)
+    out = C.c_void_p()
+    rc = lib().shingle_graph_create(n, nnz, _addr(row_ptr), _addr(col), flags, dptr, C.byref(out))
+    _check(rc)
+    return out
+
+
+def shingle_pass(h, s: int, c: int, seed: int):
+    _check(lib().shingle_pass(h, s, c, seed & 0xFFFFFFFFFFFFFFFF), h)
+
+
+def group_by_shingle(h):
+    _check(lib().group_by_shingle(h), h)
+
+
+def report_dense_subgraphs(h, mode: int = 0, min_size: int = 1, n: Optional[int] = None):
+    if n is None:
+        n = sg_get_counts(h)["n"]
+    labels = np.zeros(n, np.int32)
+    nc = C.c_int64()
+    _check(lib().report_dense_subgraphs(h, mode, min_size, labels.ctypes.data, C.byref(nc)), h)
+    return labels, nc.value
+
+
+def shingle_graph_reset(h):
+    _check(lib().shingle_graph_reset(h), h)
+
+
+def shingle_graph_destroy(h):
+    lib().shingle_graph_destroy(h)
+
+
+def sg_get_counts(h) -> dict:
+    a = np.zeros(12, np.int64)
+    _check(lib().sg_get_counts(h, a.ctypes.data), h)
+    keys = ["n", "row_lo", "rows", "n_e", "groups1", "s1p", "groups2", "pairs1", "pairs2", "state",
+            "entries2", "launches"]
+    return dict(zip(keys, (int(x) for x in a)))
+
+
+def sg_get_shingles(h, level: int):
+    rows, c = C.c_int64(), C.c_int32()
+    _check(lib().sg_get_shingles(h, level, None, None, 0, C.byref(rows), C.byref(c)), h)
+    ids = np.zeros((rows.value, c.value), np.uint64)
+    rowid = np.zeros(rows.value, np.uint32)
+    _check(lib().sg_get_shingles(h, level, ids.ctypes.data, rowid.ctypes.data, rows.value,
+                                 C.byref(rows), C.byref(c)), h)
+    return ids, rowid
+
+
+def sg_get_groups(h, level: int, with_ids: bool = True):
+    cnt = np.zeros(3, np.int64)
+    _check(lib().sg_get_groups(h, level, None, None, None, None, None, cnt.ctypes.data), h)
+    G, npairs, c = (int(x) for x in cnt)
+    tg = np.zeros(c + 1, np.int64)
+    ids = np.zeros(G, np.uint64)
+    offs = np.zeros(G + 1, np.int64)
+    mem = np.zeros(npairs, np.uint32)
+    caps = np.array([G, npairs], np.int64)
+    _check(lib().sg_get_groups(h, level, tg.ctypes.data, ids.ctypes.data if with_ids else None,
+                               offs.ctypes.data, mem.ctypes.data, caps.ctypes.data,
+                               cnt.ctypes.data), h)
+    return tg, (ids if with_ids else None), offs, mem
+
+
+def sg_get_s1p(h):
+    cnt, k0 = C.c_int64(), C.c_int64()
+    _check(lib().sg_get_s1p(h, None, 0, C.byref(cnt), C.byref(k0)), h)
+    out = np.zeros(cnt.value, np.int64)
+    _check(lib().sg_get_s1p(h, out.ctypes.data, cnt.value, C.byref(cnt), C.byref(k0)), h)
+    return out, k0.value
+
+
+def sg_get_hash_params(h, level: int, c: int):
+    A = np.zeros(c, np.uint32)
+    B = np.zeros(c, np.uint32)
+    _check(lib().sg_get_hash_params(h, level, A.ctypes.data, B.ctypes.data, c), h)
+    return A, B
+
+
+def sg_get_stage_ms(h) -> dict:
+    ms = np.zeros(len(STAGES), np.float32)
+    n = C.c_int32()
+    _check(lib().sg_get_stage_ms(h, ms.ctypes.data, len(STAGES), C.byref(n)), h)
+    return {k: float(v) for k, v in zip(STAGES, ms[: n.value])}
+
+
+def sg_partition_rows(row_ptr, world: int, kappa: int = 8) -> np.ndarray:
+    row_ptr = np.ascontiguousarray(row_ptr, np.int64)
+    b = np.zeros(world + 1, np.int64)
+    _check(lib().sg_partition_rows(len(row_ptr) - 1, row_ptr.ctypes.data, world, kappa, b.ctypes.data))
+    return b
+
+
+def sg_loopback_create(world: int):
+    out = C.c_void_p()
+    _check(lib().sg_loopback_create(world, C.byref(out)))
+    return out
+
+
+def sg_loopback_destroy(lb):
+    lib().sg_loopback_destroy(lb)
+
+
+def sg_version() -> str:
+    return lib().sg_version().decode()
+
+
+# ------------------------------------------------------------------ convenience
+class ShingleGraph:
+    """RAII wrapper: create -> pass -> group -> pass -> group -> report."""
+
+    def __init__(self, row_ptr, col, validate=True, dist=None):
+        self.h = shingle_graph_create(row_ptr, col, validate=validate, dist=dist)
+        self.n = int(row_ptr.shape[0]) - 1
+
+    def run(self, s1, c1, seed1, s2, c2, seed2):
+        shingle_pass(self.h, s1, c1, seed1)
+        group_by_shingle(self.h)
+        shingle_pass(self.h, s2, c2, seed2)
+        group_by_shingle(self.h)
+        return self
+
+    def report(self, mode=0, min_size=1):
+        return report_dense_subgraphs(self.h, mode, min_size, self.n)
+
+    def reset(self):
+        shingle_graph_reset(self.h)
+
+    def close(self):
+        if self.h is not None:
+            shingle_graph_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

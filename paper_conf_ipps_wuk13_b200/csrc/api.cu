@@ -1,0 +1,867 @@
+// api.cu — the C ABI of libshingle (include/shingle.h): handle lifecycle,
+// stage sequencing, device memory, timing and getters.  Every step of the
+// hot path runs in the kernels of kernels_pass.cu / kernels_group.cu; there
+// is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "exchange.h"
+#include "kernels.h"
+#include "report.h"
+#include "sg_internal.cuh"
+
+using namespace sg;
+
+namespace {
+
+thread_local std::string t_err;
+
+void set_err(sg_graph *g, const std::string &m) {
+  if (g) g->err = m;
+  t_err = m;
+}
+}  // namespace
+
+namespace sg {
+[[noreturn]] void fail(sg_graph *g, sg_status st, const std::string &m) {
+  set_err(g, m);
+  if (g && (st == SG_ECUDA || st == SG_ENCCL)) {
+    g->poison = st;
+    g->state = kPoisoned;
+  }
+  throw Fail{st};
+}
+
+void ck(sg_graph *g, cudaError_t e, const char *what) {
+  if (e != cudaSuccess) {
+    fail(g, SG_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+  }
+}
+}  // namespace sg
+
+namespace {
+
+#define CK(call) ck(g, (call), #call)
+
+void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
+  if (b.p) {
+    cudaFreeAsync(b.p, g->stream);
+    b.p = nullptr;
+    b.bytes = 0;
+  }
+  if (bytes == 0) bytes = 16;
+  void *p = nullptr;
+  cudaError_t e = cudaMallocAsync(&p, bytes, g->stream);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    char buf[128];
+    snprintf(buf, sizeof buf, "device allocation of %zu bytes failed", bytes);
+    fail(g, SG_ENOMEM, buf);
+  }
+  b.p = p;
+  b.bytes = bytes;
+}
+
+void dfree(sg_graph *g, DBuf &b) {
+  if (b.p) cudaFreeAsync(b.p, g->stream);
+  b.p = nullptr;
+  b.bytes = 0;
+}
+
+template <typename T>
+T *ptr(DBuf &b) {
+  return reinterpret_cast<T *>(b.p);
+}
+
+void sync(sg_graph *g) { CK(cudaStreamSynchronize(g->stream)); }
+
+void ev_begin(sg_graph *g, int id) {
+  if (!g->st[id].beg) {
+    CK(cudaEventCreate(&g->st[id].beg));
+    CK(cudaEventCreate(&g->st[id].end));
+  }
+  CK(cudaEventRecord(g->st[id].beg, g->stream));
+  g->st_used[id] = true;
+}
+
+void ev_end(sg_graph *g, int id) { CK(cudaEventRecord(g->st[id].end, g->stream)); }
+
+template <typename F>
+sg_status guarded(sg_graph *g, F &&f) {
+  if (!g) {
+    t_err = "null handle";
+    return SG_EINVAL;
+  }
+  if (g->state == kPoisoned) return g->poison;
+  try {
+    int dev = -1;
+    cudaGetDevice(&dev);
+    if (dev != g->device) CK(cudaSetDevice(g->device));
+    f();
+    return SG_OK;
+  } catch (const Fail &x) {
+    return x.st;
+  } catch (const std::bad_alloc &) {
+    set_err(g, "host allocation failed");
+    return SG_ENOMEM;
+  }
+}
+
+void free_pass(sg_graph *g, PassOut &p) {
+  dfree(g, p.A);
+  dfree(g, p.B);
+  dfree(g, p.rstart);
+  dfree(g, p.rlen);
+  dfree(g, p.rowid);
+  dfree(g, p.keys);
+  p = PassOut();
+}
+
+void free_groups(sg_graph *g, Groups &q) {
+  dfree(g, q.members);
+  dfree(g, q.head);
+  q = Groups();
+}
+
+// ---------------------------------------------------------------- validation
+__global__ void validate_kernel(const int64_t *rp, const int32_t *col, int64_t rows, int64_t nnz,
+                                int64_t n, int *bad) {
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < rows;
+       u += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = rp[u], b = rp[u + 1];
+    if (b < a || a < 0 || b > nnz) {
+      atomicExch(bad, 1);
+      continue;
+    }
+    for (int64_t e = a; e < b; ++e) {
+      const int32_t v = col[e];
+      if (v < 0 || (int64_t)v >= n || (e > a && v <= col[e - 1])) {
+        atomicExch(bad, 1);
+        break;
+      }
+    }
+  }
+}
+
+__global__ void rebase_kernel(int64_t *rp, int64_t n1, int64_t base) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n1;
+       i += (int64_t)gridDim.x * blockDim.x)
+    rp[i] -= base;
+}
+
+// ---------------------------------------------------------------- grouping
+struct GroupScratch {
+  DBuf chunk_start, chunk_len, chunk_trial, chunk_rank, seg, trial_chunk0;
+  DBuf counts, bstart, bsize, bkeys, bvals, big_list, big_count;
+};
+
+void run_group(sg_graph *g, int level, const uint64_t *keys, const uint32_t *vals,
+               const uint32_t *rowid, uint32_t val_base, const std::vector<int64_t> &seg,
+               int32_t c, Groups &out, int st_hist, int st_scatter, int st_local) {
+  const int64_t npairs = seg[(size_t)c];
+  int64_t maxseg = 0;
+  for (int j = 0; j < c; ++j) maxseg = std::max(maxseg, seg[(size_t)j + 1] - seg[(size_t)j]);
+  if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
+  int bits = 0;
+  while ((maxseg >> bits) > 1024 && bits < 14) ++bits;
+  const int64_t nbins = (int64_t)1 << bits;
+  const int64_t CH = std::max<int64_t>(8192, 8 * nbins);
+  std::vector<int64_t> cst;
+  std::vector<int32_t> clen, ctr, crk, tc0((size_t)c + 1);
+  for (int j = 0; j < c; ++j) {
+    tc0[(size_t)j] = (int32_t)cst.size();
+    int r = 0;
+    for (int64_t a = seg[(size_t)j]; a < seg[(size_t)j + 1]; a += CH) {
+      cst.push_back(a);
+      clen.push_back((int32_t)std::min<int64_t>(CH, seg[(size_t)j + 1] - a));
+      ctr.push_back(j);
+      crk.push_back(r++);
+    }
+  }
+  tc0[(size_t)c] = (int32_t)cst.size();
+  const int64_t nch = (int64_t)cst.size();
+
+  GroupScratch S;
+  auto up = [&](DBuf &b, const void *h, size_t bytes) {
+    dalloc(g, b, bytes);
+    if (bytes) CK(cudaMemcpyAsync(b.p, h, bytes, cudaMemcpyHostToDevice, g->stream));
+  };
+  up(S.chunk_start, cst.data(), cst.size() * 8);
+  up(S.chunk_len, clen.data(), clen.size() * 4);
+  up(S.chunk_trial, ctr.data(), ctr.size() * 4);
+  up(S.chunk_rank, crk.data(), crk.size() * 4);
+  up(S.seg, seg.data(), seg.size() * 8);
+  up(S.trial_chunk0, tc0.data(), tc0.size() * 4);
+  dalloc(g, S.counts, (size_t)(nch * nbins) * 4);
+  dalloc(g, S.bstart, (size_t)(c * nbins) * 4);
+  dalloc(g, S.bsize, (size_t)(c * nbins) * 4);
+  dalloc(g, S.bkeys, (size_t)npairs * 8);
+  dalloc(g, S.bvals, (size_t)npairs * 4);
+  dalloc(g, S.big_list, (size_t)(c * nbins) * 4);
+  dalloc(g, S.big_count, 4);
+  free_groups(g, out);
+  out.c = c;
+  out.npairs = npairs;
+  out.seg = seg;
+  dalloc(g, out.members, (size_t)npairs * 4);
+  dalloc(g, out.head, (size_t)((npairs + 31) / 32) * 4);
+  CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
+  CK(cudaMemsetAsync(S.big_count.p, 0, 4, g->stream));
+  // NOTE: the uploads above are tiny (per-chunk tables), not per-pair data.
+  GroupArgs a;
+  a.plan.c = c;
+  a.plan.bits = bits;
+  a.plan.nbins = nbins;
+  a.plan.nchunks = nch;
+  a.plan.npairs = npairs;
+  a.plan.chunk_start = ptr<int64_t>(S.chunk_start);
+  a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
+  a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
+  a.plan.chunk_rank = ptr<int32_t>(S.chunk_rank);
+  a.plan.seg = ptr<int64_t>(S.seg);
+  a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
+  a.keys = keys;
+  a.vals = vals;
+  a.rowid = rowid;
+  a.val_base = val_base;
+  a.counts = ptr<uint32_t>(S.counts);
+  a.bstart = ptr<uint32_t>(S.bstart);
+  a.bsize = ptr<uint32_t>(S.bsize);
+  a.bkeys = ptr<uint64_t>(S.bkeys);
+  a.bvals = ptr<uint32_t>(S.bvals);
+  a.big_list = ptr<uint32_t>(S.big_list);
+  a.big_count = ptr<uint32_t>(S.big_count);
+  a.members = ptr<uint32_t>(out.members);
+  a.head = ptr<uint32_t>(out.head);
+  ev_begin(g, st_hist);
+  CK(group_hist(a, g->stream));
+  CK(group_offsets(a, g->stream));
+  ev_end(g, st_hist);
+  ev_begin(g, st_scatter);
+  CK(group_scatter(a, g->stream));
+  ev_end(g, st_scatter);
+  ev_begin(g, st_local);
+  CK(group_local(a, g->stream));
+  uint32_t nbig = 0;
+  CK(cudaMemcpyAsync(&nbig, S.big_count.p, 4, cudaMemcpyDeviceToHost, g->stream));
+  sync(g);
+  CK(group_big(a, nbig, g->stream));
+  ev_end(g, st_local);
+  (void)level;
+  for (DBuf *b : {&S.chunk_start, &S.chunk_len, &S.chunk_trial, &S.chunk_rank, &S.seg,
+                  &S.trial_chunk0, &S.counts, &S.bstart, &S.bsize, &S.bkeys, &S.bvals,
+                  &S.big_list, &S.big_count})
+    dfree(g, *b);
+}
+
+int64_t count_groups(sg_graph *g, Groups &q) {
+  if (q.npairs == 0) return 0;
+  DBuf d;
+  dalloc(g, d, 8);
+  CK(popcount_words(ptr<uint32_t>(q.head), (q.npairs + 31) / 32,
+                    ptr<unsigned long long>(d), g->stream));
+  unsigned long long h = 0;
+  CK(cudaMemcpyAsync(&h, d.p, 8, cudaMemcpyDeviceToHost, g->stream));
+  sync(g);
+  dfree(g, d);
+  return (int64_t)h;
+}
+
+template <typename T>
+std::vector<T> d2h(sg_graph *g, const DBuf &b, size_t count) {
+  std::vector<T> v(count);
+  if (count) {
+    CK(cudaMemcpyAsync(v.data(), b.p, count * sizeof(T), cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+  }
+  return v;
+}
+
+// Host view of a grouped level: per-trial group ranges, group offsets, ids.
+struct HostGroups {
+  std::vector<int64_t> trial_goffs, offs;
+  std::vector<uint64_t> ids;
+  std::vector<uint32_t> members;
+};
+
+void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
+  Groups &q = g->grp[level];
+  PassOut &p = g->pass[level];
+  const int c = q.c;
+  H.members = d2h<uint32_t>(g, q.members, (size_t)q.npairs);
+  std::vector<uint32_t> head = d2h<uint32_t>(g, q.head, (size_t)((q.npairs + 31) / 32));
+  H.trial_goffs.assign((size_t)c + 1, 0);
+  H.offs.clear();
+  int j = 0;
+  for (int64_t i = 0; i < q.npairs; ++i) {
+    while (j < c && q.seg[(size_t)j + 1] <= i) {
+      ++j;
+      H.trial_goffs[(size_t)j] = (int64_t)H.offs.size();
+    }
+    if ((head[(size_t)(i >> 5)] >> (i & 31)) & 1u) H.offs.push_back(i);
+  }
+  while (j < c) {
+    ++j;
+    H.trial_goffs[(size_t)j] = (int64_t)H.offs.size();
+  }
+  const int64_t G = (int64_t)H.offs.size();
+  H.offs.push_back(q.npairs);
+  if (!want_ids) return;
+  // id of a group = the shingle of its first generator in that trial
+  std::vector<uint64_t> keys = d2h<uint64_t>(g, p.keys, (size_t)(p.nrows * p.c));
+  std::vector<int64_t> rowof;
+  if (level == 0) {
+    std::vector<uint32_t> rid = d2h<uint32_t>(g, p.rowid, (size_t)p.nrows);
+    rowof.assign((size_t)g->n, -1);
+    for (int64_t r = 0; r < p.nrows; ++r) rowof[rid[(size_t)r]] = r;
+  }
+  H.ids.resize((size_t)G);
+  for (int jj = 0; jj < c; ++jj) {
+    for (int64_t x = H.trial_goffs[(size_t)jj]; x < H.trial_goffs[(size_t)jj + 1]; ++x) {
+      const uint32_t m = H.members[(size_t)H.offs[(size_t)x]];
+      const int64_t r = level == 0 ? rowof[m] : (int64_t)m - g->s1p_k0;
+      H.ids[(size_t)x] = fmix_inv(keys[(size_t)(jj * p.nrows + r)]);
+    }
+  }
+}
+
+}  // namespace
+
+// =============================================================================
+extern "C" {
+
+const char *sg_version(void) { return "libshingle 0.1 (sm_100a)"; }
+
+const char *sg_last_error(const sg_graph *g) { return g ? g->err.c_str() : t_err.c_str(); }
+
+sg_status sg_partition_rows(int64_t n, const int64_t *row_ptr, int32_t world, int64_t kappa,
+                            int64_t *bounds) {
+  if (n < 0 || world < 1 || !row_ptr || !bounds) return SG_EINVAL;
+  // balance sum(deg + kappa): bounds[r] = first row whose prefix weight
+  // reaches r/world of the total
+  const long double tot = (long double)row_ptr[n] + (long double)kappa * (long double)n;
+  bounds[0] = 0;
+  int64_t u = 0;
+  for (int32_t r = 1; r < world; ++r) {
+    const long double target = tot * r / world;
+    while (u < n && (long double)row_ptr[u] + (long double)kappa * u < target) ++u;
+    bounds[r] = u;
+  }
+  bounds[world] = n;
+  return SG_OK;
+}
+
+sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col,
+                               uint32_t flags, const sg_dist *dist, sg_graph **out) {
+  if (!out) {
+    t_err = "out is NULL";
+    return SG_EINVAL;
+  }
+  *out = nullptr;
+  if (n < 0 || (uint64_t)n >= kP || nnz < 0 || (n > 0 && !row_ptr) || (nnz > 0 && !col)) {
+    t_err = "invalid n / nnz / pointers (need 0 <= n < 2^31 - 1)";
+    return SG_EINVAL;
+  }
+  if (dist && (dist->world < 1 || dist->rank < 0 || dist->rank >= dist->world)) {
+    t_err = "invalid sg_dist rank/world";
+    return SG_EINVAL;
+  }
+  const bool devptr = flags & SG_DEVICE_PTRS;
+  const bool validate = !(flags & SG_NO_VALIDATE);
+  std::vector<int64_t> hrp;
+  const int64_t *rp_host = row_ptr;
+  if (devptr && n > 0) {
+    // the partition needs the row pointers on the host (n+1 words, untimed)
+    hrp.resize((size_t)n + 1);
+    if (cudaMemcpy(hrp.data(), row_ptr, (n + 1) * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      cudaGetLastError();
+      t_err = "cannot read device row_ptr";
+      return SG_EINVAL;
+    }
+    rp_host = hrp.data();
+  }
+  if (n > 0 && (rp_host[0] != 0 || rp_host[n] != nnz)) {
+    t_err = "invalid CSR: row_ptr[0] must be 0 and row_ptr[n] must equal nnz";
+    return SG_EINVAL;
+  }
+  std::unique_ptr<sg_graph> G(new sg_graph());
+  sg_graph *g = G.get();
+  g->n = n;
+  g->nnz_global = nnz;
+  g->rank = dist ? dist->rank : 0;
+  g->world = dist ? dist->world : 1;
+  sg_status st = SG_OK;
+  try {
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+      cudaGetLastError();
+      fail(g, SG_ECUDA, "no CUDA device available (libshingle has no CPU fallback)");
+    }
+    if (dist) g->device = dist->device;
+    else CK(cudaGetDevice(&g->device));
+    CK(cudaSetDevice(g->device));
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, g->device));
+    g->num_sms = prop.multiProcessorCount;
+    if (dist && dist->stream) {
+      g->stream = (cudaStream_t)dist->stream;
+    } else {
+      CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+      g->own_stream = true;
+    }
+    // keep freed blocks cached in the pool: re-runs and resets reuse them
+    cudaMemPool_t pool;
+    CK(cudaDeviceGetDefaultMemPool(&pool, g->device));
+    uint64_t thr = UINT64_MAX;
+    CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    // row range of this rank
+    std::vector<int64_t> bounds((size_t)g->world + 1);
+    if (n > 0) sg_partition_rows(n, rp_host, g->world, 8, bounds.data());
+    else std::fill(bounds.begin(), bounds.end(), 0);
+    g->row_lo = bounds[(size_t)g->rank];
+    g->row_hi = bounds[(size_t)g->rank + 1];
+    const int64_t rows = g->row_hi - g->row_lo;
+    const int64_t e0 = n > 0 ? rp_host[g->row_lo] : 0;
+    const int64_t e1 = n > 0 ? rp_host[g->row_hi] : 0;
+    g->nnz_local = e1 - e0;
+    dalloc(g, g->row_ptr, (size_t)(rows + 1) * 8);
+    dalloc(g, g->col, (size_t)g->nnz_local * 4);
+    const cudaMemcpyKind kind = devptr ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+    if (n > 0) {
+      CK(cudaMemcpyAsync(g->row_ptr.p, row_ptr + g->row_lo, (rows + 1) * 8, kind, g->stream));
+      if (g->nnz_local)
+        CK(cudaMemcpyAsync(g->col.p, col + e0, g->nnz_local * 4, kind, g->stream));
+      rebase_kernel<<<std::min<int64_t>((rows + 256) / 256, 4096), 256, 0, g->stream>>>(
+          ptr<int64_t>(g->row_ptr), rows + 1, e0);
+      CK(cudaGetLastError());
+    } else {
+      CK(cudaMemsetAsync(g->row_ptr.p, 0, 8, g->stream));
+    }
+    if (validate && rows > 0) {
+      // the CSR is validated on the device after the copy (O(nnz), one pass)
+      DBuf bad;
+      dalloc(g, bad, 4);
+      CK(cudaMemsetAsync(bad.p, 0, 4, g->stream));
+      validate_kernel<<<std::min<int64_t>((rows + 255) / 256, 8192), 256, 0, g->stream>>>(
+          ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col.p), rows,
+          g->nnz_local, n, ptr<int>(bad));
+      CK(cudaGetLastError());
+      int hb = 0;
+      CK(cudaMemcpyAsync(&hb, bad.p, 4, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      dfree(g, bad);
+      if (hb) fail(g, SG_EINVAL, "invalid CSR: a row is not strictly increasing, or an id is outside [0, n)");
+    }
+    if (g->world > 1) {
+      g->xch = exchange_create(g, dist);
+    }
+    sync(g);
+    g->launch_base = g_launches.load();
+    g->state = kCreated;
+  } catch (const Fail &f) {
+    st = f.st;
+    t_err = g->err;
+  }
+  if (st != SG_OK) {
+    if (g->xch) exchange_destroy(g->xch);
+    for (DBuf *b : {&g->row_ptr, &g->col})
+      if (b->p) cudaFree(b->p);
+    if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+    return st;
+  }
+  *out = G.release();
+  return SG_OK;
+}
+
+sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
+  return guarded(g, [&] {
+    if (s < 1 || s > kMaxS || c < 1 || c > kMaxC) fail(g, SG_EINVAL, "need 1 <= s <= 8 and 1 <= c <= 1024");
+    int level;
+    if (g->state == kCreated) level = 0;
+    else if (g->state == kGrouped1) level = 1;
+    else fail(g, SG_ESTATE, "shingle_pass: call create -> pass -> group -> pass -> group");
+    PassOut &P = g->pass[level];
+    free_pass(g, P);
+    P.s = s;
+    P.c = c;
+    P.seed = seed;
+    P.hA.resize((size_t)c);
+    P.hB.resize((size_t)c);
+    hash_pairs(seed, c, P.hA.data(), P.hB.data());
+    const int st_all = level == 0 ? kStPass1 : kStPass2;
+    ev_begin(g, st_all);
+    ev_begin(g, level == 0 ? kStSelect1 : kStSelect2);
+    dalloc(g, P.A, (size_t)c * 4);
+    dalloc(g, P.B, (size_t)c * 4);
+    CK(cudaMemcpyAsync(P.A.p, P.hA.data(), (size_t)c * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(cudaMemcpyAsync(P.B.p, P.hB.data(), (size_t)c * 4, cudaMemcpyHostToDevice, g->stream));
+    // ---- rows
+    DBuf blk, tot;
+    int64_t nrows = 0;
+    const uint32_t *entries;
+    if (level == 0) {
+      const int64_t rows = g->row_hi - g->row_lo;
+      dalloc(g, blk, (size_t)sel_scratch_elems(rows) * 8);
+      dalloc(g, tot, 8);
+      CK(select_csr_count(ptr<int64_t>(g->row_ptr), rows, s, ptr<int64_t>(blk), ptr<int64_t>(tot),
+                          g->stream));
+      CK(cudaMemcpyAsync(&nrows, tot.p, 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      dalloc(g, P.rstart, (size_t)nrows * 8);
+      dalloc(g, P.rlen, (size_t)nrows * 4);
+      dalloc(g, P.rowid, (size_t)nrows * 4);
+      CK(select_csr_write(ptr<int64_t>(g->row_ptr), rows, s, g->row_lo, ptr<int64_t>(blk),
+                          ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), ptr<uint32_t>(P.rowid),
+                          g->stream));
+      entries = reinterpret_cast<const uint32_t *>(g->col.p);
+    } else {
+      Groups &G1 = g->grp[0];
+      dalloc(g, blk, (size_t)sel_scratch_elems((G1.npairs + 31) / 32) * 8);
+      dalloc(g, tot, 8);
+      CK(select_groups_count(ptr<uint32_t>(G1.head), G1.npairs, s, ptr<int64_t>(blk),
+                             ptr<int64_t>(tot), g->stream));
+      CK(cudaMemcpyAsync(&nrows, tot.p, 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      dalloc(g, P.rstart, (size_t)nrows * 8);
+      dalloc(g, P.rlen, (size_t)nrows * 4);
+      CK(select_groups_write(ptr<uint32_t>(G1.head), G1.npairs, s, ptr<int64_t>(blk),
+                             ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), g->stream));
+      entries = ptr<uint32_t>(G1.members);
+    }
+    P.nrows = nrows;
+    if (nrows * (int64_t)c >= ((int64_t)1 << 40))
+      fail(g, SG_EOVERFLOW, "rows * c too large for one rank");
+    if (level == 0 && g->world > 1) {
+      exchange_row_counts(g, 0, nrows);  // n_e global, row base
+    } else if (level == 0) {
+      g->n_e_global = nrows;
+      P.row_base = 0;
+    } else if (g->world > 1) {
+      exchange_row_counts(g, 1, nrows);  // |S1'| global, k0 (canonical dense index)
+    } else {
+      g->s1p_global = nrows;
+      g->s1p_k0 = 0;
+      P.row_base = 0;
+    }
+    if (level == 1 && g->s1p_global >= (int64_t)0xFFFFFFFFll)
+      fail(g, SG_EOVERFLOW, "|S1'| exceeds 2^32 - 1 (members are u32)");
+    ev_end(g, level == 0 ? kStSelect1 : kStSelect2);
+    // ---- min-hash top-s (the hot kernel)
+    ev_begin(g, level == 0 ? kStHash1 : kStHash2);
+    dalloc(g, P.keys, (size_t)(nrows * c) * 8);
+    DBuf ctr;
+    dalloc(g, ctr, 8);
+    CK(cudaMemsetAsync(ctr.p, 0, 8, g->stream));
+    MinhashArgs a;
+    a.rstart = ptr<int64_t>(P.rstart);
+    a.rlen = ptr<int32_t>(P.rlen);
+    a.entries = entries;
+    a.nrows = nrows;
+    a.A = ptr<uint32_t>(P.A);
+    a.B = ptr<uint32_t>(P.B);
+    a.c = c;
+    a.s = s;
+    a.seed = seed;
+    a.keys = ptr<uint64_t>(P.keys);
+    a.counter = ptr<unsigned long long>(ctr);
+    CK(minhash(a, g->num_sms, g->stream));
+    ev_end(g, level == 0 ? kStHash1 : kStHash2);
+    ev_end(g, st_all);
+    dfree(g, ctr);
+    dfree(g, blk);
+    dfree(g, tot);
+    sync(g);
+    g->state = level == 0 ? kPassed1 : kPassed2;
+  });
+}
+
+sg_status group_by_shingle(sg_graph *g) {
+  return guarded(g, [&] {
+    int level;
+    if (g->state == kPassed1) level = 0;
+    else if (g->state == kPassed2) level = 1;
+    else fail(g, SG_ESTATE, "group_by_shingle: needs a completed shingle_pass");
+    PassOut &P = g->pass[level];
+    const int c = P.c;
+    ev_begin(g, level == 0 ? kStGroup1 : kStGroup2);
+    if (g->world > 1) {
+      exchange_and_group(g, level);
+    } else {
+      std::vector<int64_t> seg((size_t)c + 1);
+      for (int j = 0; j <= c; ++j) seg[(size_t)j] = (int64_t)j * P.nrows;
+      const uint32_t *rowid = level == 0 ? ptr<uint32_t>(P.rowid) : nullptr;
+      const uint32_t base = level == 0 ? 0u : (uint32_t)g->s1p_k0;
+      run_group(g, level, ptr<uint64_t>(P.keys), nullptr, rowid, base, seg, c, g->grp[level],
+                level == 0 ? kStHist1 : kStHist2, level == 0 ? kStScatter1 : kStScatter2,
+                level == 0 ? kStLocal1 : kStLocal2);
+      g->pairs_global[level] = g->grp[level].npairs;
+    }
+    ev_end(g, level == 0 ? kStGroup1 : kStGroup2);
+    sync(g);
+    g->groups_global[level] = -1;  // computed lazily by sg_get_counts
+    if (level == 1) g->e2_global = -1;
+    g->state = level == 0 ? kGrouped1 : kGrouped2;
+  });
+}
+
+sg_status shingle_graph_reset(sg_graph *g) {
+  return guarded(g, [&] {
+    for (int l = 0; l < 2; ++l) {
+      free_pass(g, g->pass[l]);
+      free_groups(g, g->grp[l]);
+    }
+    sync(g);
+    g->e2_global = -1;
+    g->launch_base = g_launches.load();
+    g->state = kCreated;
+  });
+}
+
+void shingle_graph_destroy(sg_graph *g) {
+  if (!g) return;
+  cudaSetDevice(g->device);
+  if (g->stream) cudaStreamSynchronize(g->stream);
+  for (int l = 0; l < 2; ++l) {
+    PassOut &p = g->pass[l];
+    for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid, &p.keys})
+      if (b->p) cudaFree(b->p);
+    for (DBuf *b : {&g->grp[l].members, &g->grp[l].head})
+      if (b->p) cudaFree(b->p);
+  }
+  for (DBuf *b : {&g->row_ptr, &g->col, &g->s1p_gidx, &g->scratch})
+    if (b->p) cudaFree(b->p);
+  for (int i = 0; i < kNumStages; ++i) {
+    if (g->st[i].beg) cudaEventDestroy(g->st[i].beg);
+    if (g->st[i].end) cudaEventDestroy(g->st[i].end);
+  }
+  if (g->xch) exchange_destroy(g->xch);
+  if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+  cudaGetLastError();
+  delete g;
+}
+
+sg_status sg_get_counts(const sg_graph *gc, int64_t counts[12]) {
+  sg_graph *g = const_cast<sg_graph *>(gc);
+  return guarded(g, [&] {
+    if (!counts) fail(g, SG_EINVAL, "counts is NULL");
+    const long long launches = g_launches.load() - g->launch_base;  // before getter kernels
+    for (int l = 0; l < 2; ++l) {
+      const bool grouped = g->state >= (l == 0 ? kGrouped1 : kGrouped2);
+      if (grouped && g->groups_global[l] < 0) {
+        int64_t loc = count_groups(g, g->grp[l]);
+        g->groups_global[l] = g->world > 1 ? exchange_sum(g, loc) : loc;
+      }
+    }
+    if (g->state >= kPassed2 && g->e2_global < 0) {
+      DBuf d;
+      dalloc(g, d, 8);
+      CK(sum_i32(ptr<int32_t>(g->pass[1].rlen), g->pass[1].nrows, ptr<unsigned long long>(d),
+                 g->stream));
+      unsigned long long h = 0;
+      CK(cudaMemcpyAsync(&h, d.p, 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      dfree(g, d);
+      g->e2_global = g->world > 1 ? exchange_sum(g, (int64_t)h) : (int64_t)h;
+    }
+    counts[0] = g->n;
+    counts[1] = g->row_lo;
+    counts[2] = g->row_hi - g->row_lo;
+    counts[3] = g->state >= kPassed1 ? g->n_e_global : 0;
+    counts[4] = g->state >= kGrouped1 ? g->groups_global[0] : 0;
+    counts[5] = g->state >= kPassed2 ? g->s1p_global : 0;
+    counts[6] = g->state >= kGrouped2 ? g->groups_global[1] : 0;
+    counts[7] = g->state >= kGrouped1 ? g->pairs_global[0] : 0;
+    counts[8] = g->state >= kGrouped2 ? g->pairs_global[1] : 0;
+    counts[9] = g->state;
+    counts[10] = g->state >= kPassed2 ? g->e2_global : 0;
+    counts[11] = (int64_t)launches;
+  });
+}
+
+sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *rowid,
+                          int64_t cap_rows, int64_t *rows, int32_t *c) {
+  return guarded(g, [&] {
+    if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
+    const int l = level - 1;
+    if (g->state < (l == 0 ? kPassed1 : kPassed2)) fail(g, SG_ESTATE, "pass not run yet");
+    PassOut &P = g->pass[l];
+    if (rows) *rows = P.nrows;
+    if (c) *c = P.c;
+    if (!ids && !rowid) return;
+    if (cap_rows < P.nrows) fail(g, SG_EINVAL, "buffer too small");
+    if (ids) {
+      DBuf t;
+      dalloc(g, t, (size_t)(P.nrows * P.c) * 8);
+      CK(transpose_keys_to_ids(ptr<uint64_t>(P.keys), P.nrows, P.c, ptr<uint64_t>(t), g->stream));
+      CK(cudaMemcpyAsync(ids, t.p, (size_t)(P.nrows * P.c) * 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      dfree(g, t);
+    }
+    if (rowid) {
+      if (l == 0) {
+        CK(cudaMemcpyAsync(rowid, P.rowid.p, (size_t)P.nrows * 4, cudaMemcpyDeviceToHost, g->stream));
+        sync(g);
+      } else {
+        for (int64_t r = 0; r < P.nrows; ++r) rowid[r] = (uint32_t)(g->s1p_k0 + r);
+      }
+    }
+  });
+}
+
+sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64_t *ids,
+                        int64_t *offs, uint32_t *members, const int64_t caps[2], int64_t counts[3]) {
+  return guarded(g, [&] {
+    if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
+    const int l = level - 1;
+    if (g->state < (l == 0 ? kGrouped1 : kGrouped2)) fail(g, SG_ESTATE, "not grouped yet");
+    if (g->world > 1 && ids) exchange_require_single(g, "sg_get_groups ids");
+    HostGroups H;
+    host_groups(g, l, H, ids != nullptr);
+    const int64_t G = (int64_t)H.offs.size() - 1;
+    if (counts) {
+      counts[0] = G;
+      counts[1] = (int64_t)H.members.size();
+      counts[2] = g->grp[l].c;
+    }
+    if (!trial_goffs && !ids && !offs && !members) return;
+    if (!caps || caps[0] < G || caps[1] < (int64_t)H.members.size())
+      fail(g, SG_EINVAL, "buffers too small");
+    if (trial_goffs) memcpy(trial_goffs, H.trial_goffs.data(), H.trial_goffs.size() * 8);
+    if (ids) memcpy(ids, H.ids.data(), H.ids.size() * 8);
+    if (offs) memcpy(offs, H.offs.data(), H.offs.size() * 8);
+    if (members) memcpy(members, H.members.data(), H.members.size() * 4);
+  });
+}
+
+sg_status sg_get_s1p(sg_graph *g, int64_t *s1p_group, int64_t cap, int64_t *count, int64_t *k0) {
+  return guarded(g, [&] {
+    if (g->state < kPassed2) fail(g, SG_ESTATE, "pass II not run yet");
+    PassOut &P = g->pass[1];
+    if (count) *count = P.nrows;
+    if (k0) *k0 = g->s1p_k0;
+    if (!s1p_group) return;
+    if (cap < P.nrows) fail(g, SG_EINVAL, "buffer too small");
+    std::vector<int64_t> rs = d2h<int64_t>(g, P.rstart, (size_t)P.nrows);
+    Groups &q = g->grp[0];
+    std::vector<uint32_t> head = d2h<uint32_t>(g, q.head, (size_t)((q.npairs + 31) / 32));
+    // group index of the group starting at pair rs[k] = heads before rs[k]
+    int64_t gi = -1, k = 0;
+    for (int64_t i = 0; i < q.npairs && k < P.nrows; ++i) {
+      if ((head[(size_t)(i >> 5)] >> (i & 31)) & 1u) ++gi;
+      while (k < P.nrows && rs[(size_t)k] == i) s1p_group[k++] = gi;
+    }
+  });
+}
+
+sg_status sg_get_hash_params(sg_graph *g, int32_t level, uint32_t *A, uint32_t *B, int32_t cap) {
+  return guarded(g, [&] {
+    if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
+    PassOut &P = g->pass[level - 1];
+    if (P.c == 0) fail(g, SG_ESTATE, "pass not run yet");
+    if (cap < P.c) fail(g, SG_EINVAL, "buffer too small");
+    if (A) memcpy(A, P.hA.data(), (size_t)P.c * 4);
+    if (B) memcpy(B, P.hB.data(), (size_t)P.c * 4);
+  });
+}
+
+sg_status sg_get_stage_ms(const sg_graph *gc, float *ms, int32_t cap, int32_t *n) {
+  sg_graph *g = const_cast<sg_graph *>(gc);
+  return guarded(g, [&] {
+    const int k = std::min<int>(cap, kNumStages);
+    for (int i = 0; i < k; ++i) {
+      float v = 0.f;
+      if (g->st_used[i] && ms) {
+        if (cudaEventElapsedTime(&v, g->st[i].beg, g->st[i].end) != cudaSuccess) {
+          cudaGetLastError();
+          v = 0.f;
+        }
+      }
+      if (ms) ms[i] = v;
+    }
+    if (n) *n = k;
+  });
+}
+
+sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
+                                 int64_t *n_clusters) {
+  return guarded(g, [&] {
+    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
+    if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
+    if (g->world > 1) exchange_require_single(g, "report_dense_subgraphs");
+    PassOut &P1 = g->pass[0];
+    PassOut &P2 = g->pass[1];
+    HostGroups H1, H2;
+    host_groups(g, 0, H1, true);
+    host_groups(g, 1, H2, true);
+    // S1' nodes: pass-II rows, in order; group of row k starts at rstart[k]
+    std::vector<int64_t> rs = d2h<int64_t>(g, P2.rstart, (size_t)P2.nrows);
+    std::vector<int32_t> rl = d2h<int32_t>(g, P2.rlen, (size_t)P2.nrows);
+    const int64_t nk = P2.nrows;
+    std::vector<int32_t> trial1((size_t)nk);
+    std::vector<uint64_t> id1((size_t)nk);
+    std::vector<int64_t> loff((size_t)nk + 1);
+    {
+      size_t gi = 0;
+      int j = 0;
+      for (int64_t k = 0; k < nk; ++k) {
+        while (H1.offs[gi] < rs[(size_t)k]) ++gi;
+        while (g->grp[0].seg[(size_t)j + 1] <= rs[(size_t)k]) ++j;
+        trial1[(size_t)k] = j;
+        id1[(size_t)k] = H1.ids[gi];
+        loff[(size_t)k] = rs[(size_t)k];
+      }
+      loff[(size_t)nk] = nk ? rs[(size_t)nk - 1] + rl[(size_t)nk - 1] : 0;
+    }
+    // L(k) = members[rs[k] .. rs[k] + rl[k]) — build a compact copy
+    std::vector<int64_t> lo2((size_t)nk + 1, 0);
+    std::vector<uint32_t> lm;
+    lm.reserve((size_t)(nk * 4));
+    for (int64_t k = 0; k < nk; ++k) {
+      lo2[(size_t)k] = (int64_t)lm.size();
+      lm.insert(lm.end(), H1.members.begin() + rs[(size_t)k],
+                H1.members.begin() + rs[(size_t)k] + rl[(size_t)k]);
+    }
+    lo2[(size_t)nk] = (int64_t)lm.size();
+    const int64_t nh = (int64_t)H2.offs.size() - 1;
+    std::vector<int32_t> trial2((size_t)nh);
+    for (int t = 0; t < g->grp[1].c; ++t)
+      for (int64_t h = H2.trial_goffs[(size_t)t]; h < H2.trial_goffs[(size_t)t + 1]; ++h)
+        trial2[(size_t)h] = t;
+    std::vector<int64_t> hrp;
+    std::vector<int32_t> hcol;
+    if (P1.s >= 3) {
+      hrp = d2h<int64_t>(g, g->row_ptr, (size_t)(g->row_hi - g->row_lo + 1));
+      hcol = d2h<int32_t>(g, g->col, (size_t)g->nnz_local);
+    }
+    ReportInput in;
+    in.n = g->n;
+    in.s1 = P1.s;
+    in.s2 = P2.s;
+    in.A1 = P1.hA.data();
+    in.B1 = P1.hB.data();
+    in.A2 = P2.hA.data();
+    in.B2 = P2.hB.data();
+    in.nk = nk;
+    in.trial1 = trial1.data();
+    in.id1 = id1.data();
+    in.loff = lo2.data();
+    in.lmem = lm.data();
+    in.nh = nh;
+    in.trial2 = trial2.data();
+    in.id2 = H2.ids.data();
+    in.koff = H2.offs.data();
+    in.kmem = H2.members.data();
+    in.row_ptr = hrp.empty() ? nullptr : hrp.data();
+    in.col = hcol.empty() ? nullptr : hcol.data();
+    const int64_t nc = report_host(in, mode, min_size, labels);
+    if (n_clusters) *n_clusters = nc;
+  });
+}
+
+}  // extern "C"

@@ -1,0 +1,96 @@
+// kernels.h — host launchers of the libshingle device kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+namespace sg {
+
+// Number of device-kernel launches issued by this library (process-wide).
+extern std::atomic<long long> g_launches;
+
+// ---- row selection (kernels_pass.cu) ---------------------------------------
+// Pass I rows: local CSR rows with deg >= s.  Two launches with a
+// host read of the count in between (the count sizes the next allocations).
+// `blk` is device scratch of sel_scratch_elems(nrows_local) int64.
+int64_t sel_scratch_elems(int64_t items);
+cudaError_t select_csr_count(const int64_t *row_ptr, int64_t nrows_local, int s, int64_t *blk,
+                             int64_t *d_total, cudaStream_t st);
+cudaError_t select_csr_write(const int64_t *row_ptr, int64_t nrows_local, int s, int64_t row_lo,
+                             const int64_t *blk, int64_t *rstart, int32_t *rlen, uint32_t *rowid,
+                             cudaStream_t st);
+// Pass II rows: groups of G_I (head bits over npairs members) with |L| >= s
+// (S1'), in canonical order.
+cudaError_t select_groups_count(const uint32_t *head, int64_t npairs, int s, int64_t *blk,
+                                int64_t *d_total, cudaStream_t st);
+cudaError_t select_groups_write(const uint32_t *head, int64_t npairs, int s, const int64_t *blk,
+                                int64_t *rstart, int32_t *rlen, cudaStream_t st);
+
+// ---- min-hash top-s (kernels_pass.cu) --------------------------------------
+struct MinhashArgs {
+  const int64_t *rstart;
+  const int32_t *rlen;
+  const uint32_t *entries;
+  int64_t nrows;
+  const uint32_t *A;
+  const uint32_t *B;
+  int32_t c;
+  int32_t s;
+  uint64_t seed;
+  uint64_t *keys;                 // [c][nrows]
+  unsigned long long *counter;    // zeroed device counter
+};
+cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st);
+
+// ---- grouping (kernels_group.cu) -------------------------------------------
+struct GroupPlan {
+  int32_t c = 0;
+  int32_t bits = 0;          // B: bins per trial = 2^B
+  int64_t nbins = 1;
+  int64_t nchunks = 0;
+  int64_t npairs = 0;
+  // device tables
+  int64_t *chunk_start = nullptr;  // [nchunks] global pair index
+  int32_t *chunk_len = nullptr;    // [nchunks]
+  int32_t *chunk_trial = nullptr;  // [nchunks]
+  int32_t *chunk_rank = nullptr;   // [nchunks] index of the chunk within its trial
+  int64_t *seg = nullptr;          // [c+1] trial segment offsets
+  int32_t *trial_chunk0 = nullptr; // [c+1] first chunk of each trial
+};
+
+struct GroupArgs {
+  GroupPlan plan;
+  const uint64_t *keys;        // [npairs] pre-group keys (per-trial segments)
+  const uint32_t *vals;        // explicit generator values, or nullptr:
+  const uint32_t *rowid;       //   val = rowid[i - seg[j]] if rowid, else
+  uint32_t val_base;           //   val = val_base + (i - seg[j])
+  // scratch (device)
+  uint32_t *counts;            // [nchunks][nbins]
+  uint32_t *bstart;            // [c][nbins] bucket start within trial segment
+  uint32_t *bsize;             // [c][nbins]
+  uint64_t *bkeys;             // [npairs]
+  uint32_t *bvals;             // [npairs]
+  uint32_t *big_list;          // [c*nbins] bucket ids with size > local capacity
+  uint32_t *big_count;         // [1]
+  // outputs
+  uint32_t *members;           // [npairs]
+  uint32_t *head;              // [(npairs+31)/32], zeroed by the launcher
+};
+
+int64_t group_local_capacity();
+cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_scatter(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_local(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_big(const GroupArgs &g, uint32_t nbig, cudaStream_t st);
+
+// ---- getters (kernels_group.cu) --------------------------------------------
+cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
+                           cudaStream_t st);
+cudaError_t sum_i32(const int32_t *a, int64_t n, unsigned long long *d_out, cudaStream_t st);
+cudaError_t transpose_keys_to_ids(const uint64_t *keys, int64_t nrows, int32_t c, uint64_t *ids,
+                                  cudaStream_t st);
+
+}  // namespace sg

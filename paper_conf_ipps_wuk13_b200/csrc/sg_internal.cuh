@@ -1,0 +1,160 @@
+// sg_internal.cuh — internal definitions of libshingle (B200 / sm_100a).
+//
+// Product code: shares nothing with oracle/ (test infrastructure).  All
+// arithmetic here is restated from the paper and DESIGN.md's readings.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/shingle.h"
+
+namespace sg {
+
+// P = 2^31 - 1, "a big prime number" (AMB-1).
+constexpr uint32_t kP = 0x7FFFFFFFu;
+constexpr int kMaxS = 8;        // s bound of the ABI
+constexpr int kMaxC = 1024;     // c bound of the ABI
+
+// ----------------------------------------------------------------------------
+// 64-bit mixing: the splitmix64 finaliser and its inverse (bijection on 2^64).
+// Used for (a) the hash-pair stream (AMB-2), (b) the s >= 3 shingle fold
+// (AMB-4), (c) the grouping key key = fmix(id) (AMB-19).
+// ----------------------------------------------------------------------------
+__host__ __device__ __forceinline__ uint64_t fmix(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+  z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+  return z ^ (z >> 31);
+}
+
+__host__ __device__ __forceinline__ uint64_t unxorshift(uint64_t z, int s) {
+  uint64_t x = z;
+  for (int i = 0; i < 64 / s + 1; ++i) x = z ^ (x >> s);
+  return x;
+}
+
+__host__ __device__ __forceinline__ uint64_t fmix_inv(uint64_t z) {
+  z = unxorshift(z, 31);
+  z *= 0x319642b2d24d8ec3ull;   // inverse of 0x94d049bb133111eb mod 2^64
+  z = unxorshift(z, 27);
+  z *= 0x96de1b173f119089ull;   // inverse of 0xbf58476d1ce4e5b9 mod 2^64
+  return unxorshift(z, 30);
+}
+
+// (A*v + B) mod (2^31 - 1) with one 32x32->64 multiply-add and a Mersenne
+// fold: t < 2^62, x = (t & P) + (t >> 31) < 2P (t <= (P-1)P), so one
+// conditional subtract finishes.  The unsigned min picks x or x - P.
+__device__ __forceinline__ uint32_t m31_hash(uint32_t A, uint32_t B, uint32_t v) {
+  uint64_t t = (uint64_t)A * v + B;
+  uint32_t lo = (uint32_t)t & kP;
+  uint32_t hi = (uint32_t)(t >> 31);
+  uint32_t x = lo + hi;
+  uint32_t y = x - kP;
+  return x < y ? x : y;
+}
+
+// ----------------------------------------------------------------------------
+// Handle
+// ----------------------------------------------------------------------------
+enum State : int32_t {
+  kCreated = 0,   // CSR resident
+  kPassed1 = 1,   // pass I keys resident
+  kGrouped1 = 2,  // G_I resident
+  kPassed2 = 3,   // pass II keys resident
+  kGrouped2 = 4,  // G_II resident
+  kPoisoned = 99
+};
+
+// Device buffer owned by the handle (stream-ordered pool allocations).
+struct DBuf {
+  void *p = nullptr;
+  size_t bytes = 0;
+};
+
+// Output of one shingling pass on this rank.
+struct PassOut {
+  int32_t s = 0, c = 0;
+  uint64_t seed = 0;
+  int64_t nrows = 0;            // local rows with >= s entries
+  int64_t row_base = 0;         // global index of this rank's first row
+  std::vector<uint32_t> hA, hB; // hash pairs (host copy)
+  DBuf A, B;                    // uint32 [c]
+  DBuf rstart;                  // int64 [nrows] first entry of each row
+  DBuf rlen;                    // int32 [nrows]
+  DBuf rowid;                   // uint32 [nrows] generator value (pass I: vertex id)
+  DBuf keys;                    // uint64 [c][nrows]  key = fmix(id), trial-major
+};
+
+// Grouped pairs of one level on this rank: per-trial segments of `members`
+// in canonical (trial, key, member) order with one head bit per group start.
+struct Groups {
+  int32_t c = 0;
+  int64_t npairs = 0;
+  int64_t ngroups = 0;                 // local group count
+  std::vector<int64_t> seg;            // [c+1] pair offsets per trial (host)
+  DBuf members;                        // uint32 [npairs]
+  DBuf keys;                           // uint64 [npairs] sorted keys (kept for ids / report)
+  DBuf head;                           // uint32 [(npairs + 31) / 32] head bits
+};
+
+struct Stage {
+  cudaEvent_t beg = nullptr, end = nullptr;
+};
+
+constexpr int kNumStages = 16;
+// stage ids
+enum StageId {
+  kStPass1 = 0, kStGroup1 = 1, kStPass2 = 2, kStGroup2 = 3,
+  kStSelect1 = 4, kStHash1 = 5, kStSelect2 = 6, kStHash2 = 7,
+  kStHist1 = 8, kStScatter1 = 9, kStLocal1 = 10,
+  kStHist2 = 11, kStScatter2 = 12, kStLocal2 = 13,
+  kStX1 = 14, kStX2 = 15
+};
+
+struct Exchange;  // multi-GPU (exchange.cu)
+
+// Error propagation inside the library: thrown by fail(), caught at the ABI.
+struct Fail {
+  sg_status st;
+};
+[[noreturn]] void fail(sg_graph *g, sg_status st, const std::string &m);
+void ck(sg_graph *g, cudaError_t e, const char *what);
+
+}  // namespace sg
+
+struct sg_graph {
+  int32_t state = sg::kCreated;
+  sg_status poison = SG_OK;
+  std::string err;
+  int32_t device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int32_t rank = 0, world = 1;
+  sg::Exchange *xch = nullptr;
+  int num_sms = 148;
+  // graph (global n; this rank's rows [row_lo, row_hi))
+  int64_t n = 0, nnz_global = 0;
+  int64_t row_lo = 0, row_hi = 0;
+  int64_t nnz_local = 0;
+  sg::DBuf row_ptr;   // int64 [rows + 1], rebased to 0
+  sg::DBuf col;       // uint32 [nnz_local]
+  // passes and groups
+  sg::PassOut pass[2];
+  sg::Groups grp[2];
+  // global counts (summed over ranks)
+  int64_t n_e_global = 0, s1p_global = 0, s1p_k0 = 0;
+  int64_t groups_global[2] = {0, 0};
+  int64_t pairs_global[2] = {0, 0};
+  int64_t e2_global = -1;       // pass-II entries (sum of |L| over S1'), lazily
+  long long launch_base = 0;    // g_launches at create / reset
+  // G_I -> S1' selection (local): group index of each local S1' node
+  sg::DBuf s1p_gidx;  // int64 [s1p_local] (only materialised for getters)
+  // stage timing
+  sg::Stage st[sg::kNumStages];
+  bool st_used[sg::kNumStages] = {};
+  // scratch
+  sg::DBuf scratch;
+};

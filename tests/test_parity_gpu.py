@@ -1,0 +1,193 @@
+"""GPU parity: libshingle (sm_100a, through the C ABI) versus the CPU oracle,
+element by element, bit-exact (all arithmetic is integer).  Covers pass-I
+shingle matrices, G_I, the S1' map, pass-II matrices, G_II and the final
+labels, across s, c, ragged tails, staging chunks, big buckets and edge cases.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from synth import graphs as SG
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def B():
+    import torch
+    torch.cuda.init()
+    from paper_conf_ipps_wuk13_b200 import binding
+    binding.lib()
+    return binding
+
+
+def run_both(B, g, s1, c1, seed1, s2, c2, seed2, report=True):
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        G.run(s1, c1, seed1, s2, c2, seed2)
+        out = dict(
+            M1=B.sg_get_shingles(G.h, 1), G1=B.sg_get_groups(G.h, 1), s1p=B.sg_get_s1p(G.h),
+            M2=B.sg_get_shingles(G.h, 2), G2=B.sg_get_groups(G.h, 2), counts=B.sg_get_counts(G.h),
+            A1=B.sg_get_hash_params(G.h, 1, c1), A2=B.sg_get_hash_params(G.h, 2, c2))
+        if report:
+            out["rep0"] = G.report(0)
+            out["rep1"] = G.report(1, 3)
+    ref = oracle.shingling(g.row_ptr, g.col, s1, c1, seed1, s2, c2, seed2)
+    return out, ref
+
+
+def assert_parity(out, ref, report=True):
+    ids1, rows1 = out["M1"]
+    assert np.array_equal(rows1, ref.rows1)
+    assert np.array_equal(ids1, ref.M1)
+    assert np.array_equal(out["A1"][0], ref.A1) and np.array_equal(out["A1"][1], ref.B1)
+    assert np.array_equal(out["A2"][0], ref.A2) and np.array_equal(out["A2"][1], ref.B2)
+    for got, want in ((out["G1"], ref.G1), (out["G2"], ref.G2)):
+        tg, ids, offs, mem = got
+        assert np.array_equal(tg, want.trial_goffs)
+        assert np.array_equal(offs, want.offs)
+        assert np.array_equal(mem, want.members)
+        assert np.array_equal(ids, want.ids)
+    s1p, k0 = out["s1p"]
+    assert k0 == 0 and np.array_equal(s1p, ref.s1p_group)
+    ids2, rows2 = out["M2"]
+    assert np.array_equal(rows2, np.arange(len(ref.s1p_group), dtype=np.uint32))
+    assert np.array_equal(ids2, ref.M2)
+    c = out["counts"]
+    assert c["n_e"] == len(ref.rows1) and c["s1p"] == len(ref.s1p_group)
+    assert c["groups1"] == len(ref.G1.ids) and c["groups2"] == len(ref.G2.ids)
+    assert c["pairs1"] == len(ref.G1.members) and c["pairs2"] == len(ref.G2.members)
+    if report:
+        l0, n0 = out["rep0"]
+        r0, m0 = ref.report(0)
+        assert n0 == m0 and np.array_equal(l0, r0)
+        l1, n1 = out["rep1"]
+        r1, m1 = ref.report(1, 3)
+        assert n1 == m1 and np.array_equal(l1, r1)
+
+
+def test_tiny_config_full_parity(B):
+    """BASELINE configs[0]: 10K vertices, ~200K edges, 50 planted cliques, s=2, c=100."""
+    g = SG.make("tiny")
+    cfg = SG.CONFIGS["tiny"]
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    assert_parity(out, ref)
+    # the 50 planted cliques are recovered as 50 of the clusters
+    assert out["rep0"][1] >= 50
+
+
+@pytest.mark.parametrize("s1,c1,s2,c2", [(1, 1, 1, 1), (1, 7, 2, 5), (2, 32, 2, 33), (3, 33, 3, 31),
+                                         (5, 20, 2, 17), (8, 9, 4, 40), (2, 64, 8, 3), (4, 100, 1, 64)])
+def test_tiny_parity_s_c_sweep(B, s1, c1, s2, c2):
+    g = SG.make("tiny")
+    out, ref = run_both(B, g, s1, c1, 1000 + c1, s2, c2, 2000 + c2)
+    assert_parity(out, ref)
+
+
+def test_small_homology_parity(B):
+    """60K vertices / 1.7M edges, same recipe as the GOS-shaped config (several
+    tiles of every kernel, ragged tails, multi-chunk histograms)."""
+    g = SG.make("small")
+    cfg = SG.CONFIGS["small"]
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    assert_parity(out, ref)
+
+
+def test_hub_rows_longer_than_staging_buffer(B):
+    """Rows of 5K-12K entries exceed the per-warp smem stage (chunked path)."""
+    g = SG.make("hubsmall")
+    assert g.degrees().max() > 4096
+    cfg = SG.CONFIGS["hubsmall"]
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    assert_parity(out, ref)
+
+
+def test_big_bucket_path_large_clique(B):
+    """A 5,000-clique: in every trial ~4,998 vertices share one shingle, a
+    group larger than the 4,096-element shared-memory bucket (global path)."""
+    g = SG.cliques([5000, 30, 12], n=6000, seed=3)
+    out, ref = run_both(B, g, 2, 6, 11, 2, 5, 12)
+    assert_parity(out, ref)
+    assert np.diff(ref.G1.offs).max() > 4096
+
+
+def test_edge_cases_empty_and_degenerate(B):
+    # no edges at all: no rows, empty groups
+    g = SG.Graph(np.zeros(51, np.int64), np.zeros(0, np.int32))
+    out, ref = run_both(B, g, 2, 10, 1, 2, 10, 2)
+    assert_parity(out, ref)
+    # a matching: every vertex has degree 1 < s = 2
+    a = np.arange(0, 40, 2)
+    g = SG.Graph(*SG._csr_from_pairs(40, a, a + 1))
+    out, ref = run_both(B, g, 2, 8, 1, 2, 8, 2)
+    assert_parity(out, ref)
+    # s = 1 on the matching: every group has |L| = 1 < s2 = 2, so S1' is empty
+    out, ref = run_both(B, g, 1, 8, 1, 2, 8, 2)
+    assert_parity(out, ref)
+    assert len(ref.s1p_group) == 0
+
+
+def test_state_machine_and_errors(B):
+    g = SG.make("tiny")
+    h = B.shingle_graph_create(g.row_ptr, g.col)
+    try:
+        with pytest.raises(B.SGError) as e:
+            B.group_by_shingle(h)
+        assert e.value.status == B.SG_ESTATE
+        with pytest.raises(B.SGError) as e:
+            B.shingle_pass(h, 9, 10, 1)
+        assert e.value.status == B.SG_EINVAL
+        with pytest.raises(B.SGError) as e:
+            B.shingle_pass(h, 2, 1025, 1)
+        assert e.value.status == B.SG_EINVAL
+        B.shingle_pass(h, 2, 10, 1)
+        with pytest.raises(B.SGError) as e:
+            B.shingle_pass(h, 2, 10, 1)
+        assert e.value.status == B.SG_ESTATE
+        with pytest.raises(B.SGError) as e:
+            B.report_dense_subgraphs(h, 0, 1, g.n)
+        assert e.value.status == B.SG_ESTATE
+    finally:
+        B.shingle_graph_destroy(h)
+
+
+def test_reset_and_rerun_identical(B):
+    g = SG.make("tiny")
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        G.run(2, 40, 5, 2, 30, 6)
+        a = B.sg_get_groups(G.h, 2)
+        G.reset()
+        G.run(2, 40, 5, 2, 30, 6)
+        b = B.sg_get_groups(G.h, 2)
+    for x, y in zip(a, b):
+        assert np.array_equal(x, y)
+
+
+def test_device_pointer_input(B):
+    import torch
+    g = SG.make("tiny")
+    rp = torch.from_numpy(g.row_ptr).cuda()
+    col = torch.from_numpy(g.col).cuda()
+    h = B.shingle_graph_create(rp, col)
+    try:
+        B.shingle_pass(h, 2, 20, 7)
+        ids, rows = B.sg_get_shingles(h, 1)
+    finally:
+        B.shingle_graph_destroy(h)
+    ref = oracle.shingling(g.row_ptr, g.col, 2, 20, 7, 2, 4, 8)
+    assert np.array_equal(rows, ref.rows1) and np.array_equal(ids, ref.M1)
+
+
+def test_invalid_csr_rejected(B):
+    g = SG.random_graph(200, 900, seed=2)
+    r = int(np.argmax(np.diff(g.row_ptr) >= 2))
+    a = g.row_ptr[r]
+    cases = []
+    bad = g.col.copy(); bad[a], bad[a + 1] = bad[a + 1], bad[a]; cases.append((g.row_ptr, bad))
+    bad = g.col.copy(); bad[a + 1] = bad[a]; cases.append((g.row_ptr, bad))
+    bad = g.col.copy(); bad[-1] = 200; cases.append((g.row_ptr, bad))
+    bad = g.col.copy(); bad[0] = -1; cases.append((g.row_ptr, bad))
+    rp = g.row_ptr.copy(); rp[-1] -= 1; cases.append((rp, g.col[:-1].copy() if False else g.col))
+    for rp, col in cases:
+        with pytest.raises(B.SGError) as e:
+            B.shingle_graph_create(rp, col)
+        assert e.value.status == B.SG_EINVAL
