@@ -140,12 +140,15 @@ SG_API const char *sg_last_error(const sg_graph *g);
 /* Getters (host buffers; two-call pattern: NULL buffers report sizes).      */
 /* ------------------------------------------------------------------------ */
 
-/* counts[0..11] = n, this rank's first row, rows on this rank, n_e (pass-I  */
+/* counts[0..15] = n, this rank's first row, rows on this rank, n_e (pass-I  */
 /* rows, global), |S1| (G_I groups), |S1'| (pass-II rows), |S2| (G_II        */
 /* groups), P1 pairs, P2 pairs, state, E2 (pass-II entries = sum of |L| over */
-/* S1'), device-kernel launches since create / the last reset.  Global      */
-/* counts are summed over ranks.                                             */
-SG_API sg_status sg_get_counts(const sg_graph *g, int64_t counts[12]);
+/* S1'), device-kernel launches since create / the last reset, trial chunks  */
+/* of pass I and of pass II (negative: keys computed inside the grouping,    */
+/* DESIGN.md §6.3), 0, 0.  Global counts are summed over ranks.  The        */
+/* environment variable SG_MEM_BUDGET (bytes, read at create) caps the HBM   */
+/* the planner assumes, to exercise the chunked paths on small graphs.      */
+SG_API sg_status sg_get_counts(const sg_graph *g, int64_t counts[16]);
 
 /* Shingle matrix of pass `level` (1 or 2) on this rank: ids[rows x c]      */
 /* row-major (rows ascending: pass I = vertices with deg >= s1 ascending;   */

@@ -144,10 +144,10 @@ def shingle_graph_destroy(h):
 
 
 def sg_get_counts(h) -> dict:
-    a = np.zeros(12, np.int64)
+    a = np.zeros(16, np.int64)
     _check(lib().sg_get_counts(h, a.ctypes.data), h)
     keys = ["n", "row_lo", "rows", "n_e", "groups1", "s1p", "groups2", "pairs1", "pairs2", "state",
-            "entries2", "launches"]
+            "entries2", "launches", "chunks1", "chunks2"]
     return dict(zip(keys, (int(x) for x in a)))
 
 

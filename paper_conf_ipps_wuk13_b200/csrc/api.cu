@@ -1,11 +1,12 @@
 // api.cu — the C ABI of libshingle (include/shingle.h): handle lifecycle,
-// stage sequencing, device memory, timing and getters.  Every step of the
-// hot path runs in the kernels of kernels_pass.cu / kernels_group.cu; there
-// is no CPU fallback.
+// stage sequencing, HBM planning, timing and getters.  Every step of the hot
+// path runs in the kernels of kernels_{pass,minhash,group}.cu; there is no
+// CPU fallback.
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <string>
@@ -19,7 +20,6 @@
 using namespace sg;
 
 namespace {
-
 thread_local std::string t_err;
 
 void set_err(sg_graph *g, const std::string &m) {
@@ -39,9 +39,7 @@ namespace sg {
 }
 
 void ck(sg_graph *g, cudaError_t e, const char *what) {
-  if (e != cudaSuccess) {
-    fail(g, SG_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
-  }
+  if (e != cudaSuccess) fail(g, SG_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 }  // namespace sg
 
@@ -52,6 +50,7 @@ namespace {
 void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
   if (b.p) {
     cudaFreeAsync(b.p, g->stream);
+    g->bytes_live -= (int64_t)b.bytes;
     b.p = nullptr;
     b.bytes = 0;
   }
@@ -60,37 +59,61 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
   cudaError_t e = cudaMallocAsync(&p, bytes, g->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
-    char buf[128];
-    snprintf(buf, sizeof buf, "device allocation of %zu bytes failed", bytes);
+    size_t fr = 0, tot = 0;
+    cudaMemGetInfo(&fr, &tot);
+    cudaGetLastError();
+    char buf[192];
+    snprintf(buf, sizeof buf, "device allocation of %zu bytes failed (device free %zu of %zu bytes)",
+             bytes, fr, tot);
     fail(g, SG_ENOMEM, buf);
   }
   b.p = p;
   b.bytes = bytes;
+  g->bytes_live += (int64_t)bytes;
 }
 
 void dfree(sg_graph *g, DBuf &b) {
-  if (b.p) cudaFreeAsync(b.p, g->stream);
+  if (b.p) {
+    cudaFreeAsync(b.p, g->stream);
+    g->bytes_live -= (int64_t)b.bytes;
+  }
   b.p = nullptr;
   b.bytes = 0;
 }
 
 template <typename T>
-T *ptr(DBuf &b) {
+T *ptr(const DBuf &b) {
   return reinterpret_cast<T *>(b.p);
 }
 
 void sync(sg_graph *g) { CK(cudaStreamSynchronize(g->stream)); }
 
-void ev_begin(sg_graph *g, int id) {
-  if (!g->st[id].beg) {
-    CK(cudaEventCreate(&g->st[id].beg));
-    CK(cudaEventCreate(&g->st[id].end));
+// ---- stage timing: CUDA events on the handle's stream ------------------------
+int ev_take(sg_graph *g) {
+  if (g->ev_next == g->ev_pool.size()) {
+    cudaEvent_t e;
+    CK(cudaEventCreate(&e));
+    g->ev_pool.push_back(e);
   }
-  CK(cudaEventRecord(g->st[id].beg, g->stream));
-  g->st_used[id] = true;
+  return (int)g->ev_next++;
 }
 
-void ev_end(sg_graph *g, int id) { CK(cudaEventRecord(g->st[id].end, g->stream)); }
+void st_begin(sg_graph *g, int id) {
+  const int e = ev_take(g);
+  CK(cudaEventRecord(g->ev_pool[(size_t)e], g->stream));
+  g->st[id].push_back({e, -1});
+}
+
+void st_end(sg_graph *g, int id) {
+  const int e = ev_take(g);
+  CK(cudaEventRecord(g->ev_pool[(size_t)e], g->stream));
+  g->st[id].back().second = e;
+}
+
+void st_clear(sg_graph *g) {
+  for (auto &v : g->st) v.clear();
+  g->ev_next = 0;
+}
 
 template <typename F>
 sg_status guarded(sg_graph *g, F &&f) {
@@ -114,12 +137,8 @@ sg_status guarded(sg_graph *g, F &&f) {
 }
 
 void free_pass(sg_graph *g, PassOut &p) {
-  dfree(g, p.A);
-  dfree(g, p.B);
-  dfree(g, p.rstart);
-  dfree(g, p.rlen);
-  dfree(g, p.rowid);
-  dfree(g, p.keys);
+  for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) dfree(g, *b);
+  for (auto &ch : p.chunks) dfree(g, ch.keys);
   p = PassOut();
 }
 
@@ -155,75 +174,182 @@ __global__ void rebase_kernel(int64_t *rp, int64_t n1, int64_t base) {
     rp[i] -= base;
 }
 
-// ---------------------------------------------------------------- grouping
-struct GroupScratch {
-  DBuf chunk_start, chunk_len, chunk_trial, chunk_rank, seg, trial_chunk0;
-  DBuf counts, bstart, bsize, bkeys, bvals, big_list, big_count;
-};
+// ---------------------------------------------------------------- HBM planning
+// Bytes the handle may still allocate: free device memory + blocks cached by
+// the stream-ordered pool, capped by the SG_MEM_BUDGET test hook.
+int64_t avail_bytes(sg_graph *g) {
+  size_t fr = 0, tot = 0;
+  CK(cudaMemGetInfo(&fr, &tot));
+  cudaMemPool_t pool;
+  CK(cudaDeviceGetDefaultMemPool(&pool, g->device));
+  uint64_t reserved = 0, used = 0;
+  CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved));
+  CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used));
+  int64_t a = (int64_t)fr + (int64_t)(reserved - used) - ((int64_t)1 << 30);
+  if (g->mem_budget > 0) a = std::min<int64_t>(a, g->mem_budget - g->bytes_live);
+  return a;
+}
 
-void run_group(sg_graph *g, int level, const uint64_t *keys, const uint32_t *vals,
-               const uint32_t *rowid, uint32_t val_base, const std::vector<int64_t> &seg,
-               int32_t c, Groups &out, int st_hist, int st_scatter, int st_local) {
-  const int64_t npairs = seg[(size_t)c];
-  int64_t maxseg = 0;
-  for (int j = 0; j < c; ++j) maxseg = std::max(maxseg, seg[(size_t)j + 1] - seg[(size_t)j]);
-  if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
-  int bits = 0;
-  while ((maxseg >> bits) > 1024 && bits < 14) ++bits;
-  const int64_t nbins = (int64_t)1 << bits;
-  const int64_t CH = std::max<int64_t>(8192, 8 * nbins);
-  std::vector<int64_t> cst;
-  std::vector<int32_t> clen, ctr, crk, tc0((size_t)c + 1);
-  for (int j = 0; j < c; ++j) {
-    tc0[(size_t)j] = (int32_t)cst.size();
-    int r = 0;
-    for (int64_t a = seg[(size_t)j]; a < seg[(size_t)j + 1]; a += CH) {
-      cst.push_back(a);
-      clen.push_back((int32_t)std::min<int64_t>(CH, seg[(size_t)j + 1] - a));
-      ctr.push_back(j);
-      crk.push_back(r++);
+// Split the c trials into chunks so that the pass's keys and the grouping's
+// scratch fit in HBM (grouping is per trial, so chunking is exact, AMB-5).
+// Eager: all keys computed by shingle_pass.  Deferred: group_by_shingle
+// computes each chunk's keys right before grouping it.
+double scratch_per_pair(int64_t maxseg);
+
+void plan_pass(sg_graph *g, PassOut &P) {
+  const int64_t nr = P.nrows, c = P.c;
+  const double keys_t = 8.0 * (double)P.key_stride;             // keys of one trial
+  const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;   // scratch per trial
+  const double members = 4.125 * (double)nr * (double)c + (1 << 20);
+  const double avail = (double)avail_bytes(g);
+  int64_t ct = (int64_t)((avail - members - keys_t * c) / scr_t);
+  P.deferred = false;
+  if (ct < 1) {
+    ct = (int64_t)((avail - members) / (keys_t + scr_t));
+    P.deferred = true;
+    if (ct < 1) {
+      char buf[160];
+      snprintf(buf, sizeof buf, "pass needs more HBM than available (%.0f B for the members alone)",
+               members);
+      fail(g, SG_ENOMEM, buf);
     }
   }
-  tc0[(size_t)c] = (int32_t)cst.size();
-  const int64_t nch = (int64_t)cst.size();
+  ct = std::min<int64_t>(ct, c);
+  const int64_t nch = (c + ct - 1) / ct;
+  const int64_t per = (c + nch - 1) / nch;
+  P.chunks.clear();
+  for (int64_t t = 0; t < c; t += per) {
+    KeyChunk k;
+    k.t0 = (int32_t)t;
+    k.nt = (int32_t)std::min<int64_t>(per, c - t);
+    P.chunks.push_back(k);
+  }
+}
 
-  GroupScratch S;
+void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
+  st_begin(g, st_hash);
+  dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
+  DBuf ctr;
+  dalloc(g, ctr, 8);
+  CK(cudaMemsetAsync(ctr.p, 0, 8, g->stream));
+  MinhashArgs a;
+  a.rstart = ptr<int64_t>(P.rstart);
+  a.rlen = ptr<int32_t>(P.rlen);
+  a.entries = P.entries;
+  a.nrows = P.nrows;
+  a.A = ptr<uint32_t>(P.A);
+  a.B = ptr<uint32_t>(P.B);
+  a.t0 = ch.t0;
+  a.nt = ch.nt;
+  a.s = P.s;
+  a.seed = P.seed;
+  a.keys = ptr<uint64_t>(ch.keys);
+  a.key_stride = P.key_stride;
+  a.counter = ptr<unsigned long long>(ctr);
+  CK(minhash(a, g->num_sms, g->stream));
+  dfree(g, ctr);
+  st_end(g, st_hash);
+  ch.computed = true;
+}
+
+// ---------------------------------------------------------------- grouping
+struct GroupScratch {
+  DBuf chunk_i0, chunk_len, chunk_trial, in_base, seg, trial_chunk0;
+  DBuf counts, bstart1, bsize1, bstart, bsize, akeys, avals, bkeys, bvals, big_list, big_count;
+};
+
+void free_scratch(sg_graph *g, GroupScratch &S) {
+  for (DBuf *b : {&S.chunk_i0, &S.chunk_len, &S.chunk_trial, &S.in_base, &S.seg, &S.trial_chunk0,
+                  &S.counts, &S.bstart1, &S.bsize1, &S.bstart, &S.bsize, &S.akeys, &S.avals,
+                  &S.bkeys, &S.bvals, &S.big_list, &S.big_count})
+    dfree(g, *b);
+}
+
+// Scratch bytes per pair of a trial segment of `maxseg` pairs (planning).
+double scratch_per_pair(int64_t maxseg) {
+  int32_t b, b1;
+  group_bits(maxseg, &b, &b1);
+  return b == b1 ? 12.5 : 24.5;
+}
+
+// Group the pairs of trials [t0, t0 + nt) whose keys are `keys` ([nt][stride])
+// into out.members / out.head at the global positions seg_all[t].
+void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, int32_t nt,
+                 const std::vector<int64_t> &seg_all, const uint32_t *vals, const uint32_t *rowid,
+                 uint32_t val_base, Groups &out, GroupScratch &S, DBuf *free_after_scatter,
+                 int st_hist, int st_scatter, int st_local) {
+  int64_t maxseg = 0, npairs = 0;
+  for (int j = 0; j < nt; ++j) {
+    const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
+    maxseg = std::max(maxseg, L);
+    npairs += L;
+  }
+  if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
+  // final buckets of ~2-4K pairs (the shared-memory sort holds 8K); the
+  // coarse scatter fans out to <= 1024 buckets, a second level splits them
+  // further for very long trial segments; chunks of >= 64 pairs per bucket
+  int32_t bits = 0, bits1 = 0;
+  group_bits(maxseg, &bits, &bits1);
+  const bool two = bits != bits1;
+  const int64_t nbins = (int64_t)1 << bits;
+  const int64_t nb1 = (int64_t)1 << bits1;
+  const int64_t CH = std::max<int64_t>(65536, 64 * nb1);
+  std::vector<int64_t> ci0, inb((size_t)nt), seg((size_t)nt + 1);
+  std::vector<int32_t> clen, ctr, tc0((size_t)nt + 1);
+  for (int j = 0; j < nt; ++j) {
+    tc0[(size_t)j] = (int32_t)ci0.size();
+    inb[(size_t)j] = (int64_t)j * stride;
+    seg[(size_t)j] = seg_all[(size_t)t0 + j];
+    const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
+    for (int64_t a = 0; a < L; a += CH) {
+      ci0.push_back(a);
+      clen.push_back((int32_t)std::min<int64_t>(CH, L - a));
+      ctr.push_back(j);
+    }
+  }
+  seg[(size_t)nt] = seg_all[(size_t)t0 + nt];
+  tc0[(size_t)nt] = (int32_t)ci0.size();
+  const int64_t nch = (int64_t)ci0.size();
   auto up = [&](DBuf &b, const void *h, size_t bytes) {
-    dalloc(g, b, bytes);
+    if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
     if (bytes) CK(cudaMemcpyAsync(b.p, h, bytes, cudaMemcpyHostToDevice, g->stream));
   };
-  up(S.chunk_start, cst.data(), cst.size() * 8);
+  auto need = [&](DBuf &b, size_t bytes) {
+    if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
+  };
+  // per-chunk tables (small host-built plans, not per-pair data)
+  up(S.chunk_i0, ci0.data(), ci0.size() * 8);
   up(S.chunk_len, clen.data(), clen.size() * 4);
   up(S.chunk_trial, ctr.data(), ctr.size() * 4);
-  up(S.chunk_rank, crk.data(), crk.size() * 4);
+  up(S.in_base, inb.data(), inb.size() * 8);
   up(S.seg, seg.data(), seg.size() * 8);
   up(S.trial_chunk0, tc0.data(), tc0.size() * 4);
-  dalloc(g, S.counts, (size_t)(nch * nbins) * 4);
-  dalloc(g, S.bstart, (size_t)(c * nbins) * 4);
-  dalloc(g, S.bsize, (size_t)(c * nbins) * 4);
-  dalloc(g, S.bkeys, (size_t)npairs * 8);
-  dalloc(g, S.bvals, (size_t)npairs * 4);
-  dalloc(g, S.big_list, (size_t)(c * nbins) * 4);
-  dalloc(g, S.big_count, 4);
-  free_groups(g, out);
-  out.c = c;
-  out.npairs = npairs;
-  out.seg = seg;
-  dalloc(g, out.members, (size_t)npairs * 4);
-  dalloc(g, out.head, (size_t)((npairs + 31) / 32) * 4);
-  CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
+  need(S.counts, (size_t)(nch * nb1) * 4);
+  need(S.bstart1, (size_t)(nt * nb1) * 4);
+  need(S.bsize1, (size_t)(nt * nb1) * 4);
+  need(S.akeys, (size_t)npairs * 8);
+  need(S.avals, (size_t)npairs * 4);
+  if (two) {
+    need(S.bstart, (size_t)(nt * nbins) * 4);
+    need(S.bsize, (size_t)(nt * nbins) * 4);
+    need(S.bkeys, (size_t)npairs * 8);
+    need(S.bvals, (size_t)npairs * 4);
+  }
+  need(S.big_list, (size_t)(nt * nbins) * 4);
+  need(S.big_count, 4);
   CK(cudaMemsetAsync(S.big_count.p, 0, 4, g->stream));
-  // NOTE: the uploads above are tiny (per-chunk tables), not per-pair data.
   GroupArgs a;
-  a.plan.c = c;
+  a.plan.c = nt;
   a.plan.bits = bits;
+  a.plan.bits1 = bits1;
   a.plan.nbins = nbins;
+  a.plan.nb1 = nb1;
   a.plan.nchunks = nch;
   a.plan.npairs = npairs;
-  a.plan.chunk_start = ptr<int64_t>(S.chunk_start);
+  a.plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
   a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
   a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
-  a.plan.chunk_rank = ptr<int32_t>(S.chunk_rank);
+  a.plan.in_base = ptr<int64_t>(S.in_base);
   a.plan.seg = ptr<int64_t>(S.seg);
   a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
   a.keys = keys;
@@ -231,41 +357,41 @@ void run_group(sg_graph *g, int level, const uint64_t *keys, const uint32_t *val
   a.rowid = rowid;
   a.val_base = val_base;
   a.counts = ptr<uint32_t>(S.counts);
-  a.bstart = ptr<uint32_t>(S.bstart);
-  a.bsize = ptr<uint32_t>(S.bsize);
-  a.bkeys = ptr<uint64_t>(S.bkeys);
-  a.bvals = ptr<uint32_t>(S.bvals);
+  a.bstart1 = ptr<uint32_t>(S.bstart1);
+  a.bsize1 = ptr<uint32_t>(S.bsize1);
+  a.akeys = ptr<uint64_t>(S.akeys);
+  a.avals = ptr<uint32_t>(S.avals);
+  a.bstart = two ? ptr<uint32_t>(S.bstart) : a.bstart1;
+  a.bsize = two ? ptr<uint32_t>(S.bsize) : a.bsize1;
+  a.bkeys = two ? ptr<uint64_t>(S.bkeys) : a.akeys;
+  a.bvals = two ? ptr<uint32_t>(S.bvals) : a.avals;
   a.big_list = ptr<uint32_t>(S.big_list);
   a.big_count = ptr<uint32_t>(S.big_count);
   a.members = ptr<uint32_t>(out.members);
   a.head = ptr<uint32_t>(out.head);
-  ev_begin(g, st_hist);
+  st_begin(g, st_hist);
   CK(group_hist(a, g->stream));
   CK(group_offsets(a, g->stream));
-  ev_end(g, st_hist);
-  ev_begin(g, st_scatter);
-  CK(group_scatter(a, g->stream));
-  ev_end(g, st_scatter);
-  ev_begin(g, st_local);
-  CK(group_local(a, g->stream));
+  st_end(g, st_hist);
+  st_begin(g, st_scatter);
+  CK(group_scatter(a, g->num_sms, g->stream));
+  if (free_after_scatter) dfree(g, *free_after_scatter);   // keys consumed
+  if (two) CK(group_scatter2(a, g->stream));
+  st_end(g, st_scatter);
+  st_begin(g, st_local);
+  CK(group_local(a, g->num_sms, g->stream));
   uint32_t nbig = 0;
   CK(cudaMemcpyAsync(&nbig, S.big_count.p, 4, cudaMemcpyDeviceToHost, g->stream));
   sync(g);
   CK(group_big(a, nbig, g->stream));
-  ev_end(g, st_local);
-  (void)level;
-  for (DBuf *b : {&S.chunk_start, &S.chunk_len, &S.chunk_trial, &S.chunk_rank, &S.seg,
-                  &S.trial_chunk0, &S.counts, &S.bstart, &S.bsize, &S.bkeys, &S.bvals,
-                  &S.big_list, &S.big_count})
-    dfree(g, *b);
+  st_end(g, st_local);
 }
 
-int64_t count_groups(sg_graph *g, Groups &q) {
-  if (q.npairs == 0) return 0;
+int64_t device_sum_popc(sg_graph *g, const DBuf &words, int64_t nwords) {
+  if (nwords == 0) return 0;
   DBuf d;
   dalloc(g, d, 8);
-  CK(popcount_words(ptr<uint32_t>(q.head), (q.npairs + 31) / 32,
-                    ptr<unsigned long long>(d), g->stream));
+  CK(popcount_words(ptr<uint32_t>(words), nwords, ptr<unsigned long long>(d), g->stream));
   unsigned long long h = 0;
   CK(cudaMemcpyAsync(&h, d.p, 8, cudaMemcpyDeviceToHost, g->stream));
   sync(g);
@@ -281,6 +407,30 @@ std::vector<T> d2h(sg_graph *g, const DBuf &b, size_t count) {
     sync(g);
   }
   return v;
+}
+
+// Recompute shingle ids of (row, trial) requests of pass `level` on device.
+std::vector<uint64_t> recompute_ids(sg_graph *g, int level, const std::vector<int64_t> &rows,
+                                    const std::vector<int32_t> &trials) {
+  PassOut &P = g->pass[level];
+  const size_t nq = rows.size();
+  std::vector<uint64_t> out(nq);
+  if (!nq) return out;
+  DBuf dr, dt, di;
+  dalloc(g, dr, nq * 8);
+  dalloc(g, dt, nq * 4);
+  dalloc(g, di, nq * 8);
+  CK(cudaMemcpyAsync(dr.p, rows.data(), nq * 8, cudaMemcpyHostToDevice, g->stream));
+  CK(cudaMemcpyAsync(dt.p, trials.data(), nq * 4, cudaMemcpyHostToDevice, g->stream));
+  CK(shingle_ids(ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), P.entries, ptr<uint32_t>(P.A),
+                 ptr<uint32_t>(P.B), P.s, P.seed, ptr<int64_t>(dr), ptr<int32_t>(dt),
+                 (int64_t)nq, ptr<uint64_t>(di), g->stream));
+  CK(cudaMemcpyAsync(out.data(), di.p, nq * 8, cudaMemcpyDeviceToHost, g->stream));
+  sync(g);
+  dfree(g, dr);
+  dfree(g, dt);
+  dfree(g, di);
+  return out;
 }
 
 // Host view of a grouped level: per-trial group ranges, group offsets, ids.
@@ -313,22 +463,20 @@ void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
   const int64_t G = (int64_t)H.offs.size();
   H.offs.push_back(q.npairs);
   if (!want_ids) return;
-  // id of a group = the shingle of its first generator in that trial
-  std::vector<uint64_t> keys = d2h<uint64_t>(g, p.keys, (size_t)(p.nrows * p.c));
-  std::vector<int64_t> rowof;
-  if (level == 0) {
-    std::vector<uint32_t> rid = d2h<uint32_t>(g, p.rowid, (size_t)p.nrows);
-    rowof.assign((size_t)g->n, -1);
-    for (int64_t r = 0; r < p.nrows; ++r) rowof[rid[(size_t)r]] = r;
-  }
-  H.ids.resize((size_t)G);
+  // id of a group = the shingle of its first (smallest) generator in that trial
+  std::vector<uint32_t> rid;
+  if (level == 0) rid = d2h<uint32_t>(g, p.rowid, (size_t)p.nrows);
+  std::vector<int64_t> rows((size_t)G);
+  std::vector<int32_t> trials((size_t)G);
   for (int jj = 0; jj < c; ++jj) {
     for (int64_t x = H.trial_goffs[(size_t)jj]; x < H.trial_goffs[(size_t)jj + 1]; ++x) {
       const uint32_t m = H.members[(size_t)H.offs[(size_t)x]];
-      const int64_t r = level == 0 ? rowof[m] : (int64_t)m - g->s1p_k0;
-      H.ids[(size_t)x] = fmix_inv(keys[(size_t)(jj * p.nrows + r)]);
+      rows[(size_t)x] = level == 0 ? (int64_t)(std::lower_bound(rid.begin(), rid.end(), m) - rid.begin())
+                                   : (int64_t)m - g->s1p_k0;
+      trials[(size_t)x] = jj;
     }
   }
+  H.ids = recompute_ids(g, level, rows, trials);
 }
 
 }  // namespace
@@ -336,7 +484,7 @@ void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
 // =============================================================================
 extern "C" {
 
-const char *sg_version(void) { return "libshingle 0.1 (sm_100a)"; }
+const char *sg_version(void) { return "libshingle 0.2 (sm_100a)"; }
 
 const char *sg_last_error(const sg_graph *g) { return g ? g->err.c_str() : t_err.c_str(); }
 
@@ -396,6 +544,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
   g->nnz_global = nnz;
   g->rank = dist ? dist->rank : 0;
   g->world = dist ? dist->world : 1;
+  if (const char *mb = getenv("SG_MEM_BUDGET")) g->mem_budget = atoll(mb);
   sg_status st = SG_OK;
   try {
     int ndev = 0;
@@ -458,9 +607,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
       dfree(g, bad);
       if (hb) fail(g, SG_EINVAL, "invalid CSR: a row is not strictly increasing, or an id is outside [0, n)");
     }
-    if (g->world > 1) {
-      g->xch = exchange_create(g, dist);
-    }
+    if (g->world > 1) g->xch = exchange_create(g, dist);
     sync(g);
     g->launch_base = g_launches.load();
     g->state = kCreated;
@@ -486,6 +633,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     if (g->state == kCreated) level = 0;
     else if (g->state == kGrouped1) level = 1;
     else fail(g, SG_ESTATE, "shingle_pass: call create -> pass -> group -> pass -> group");
+    if (level == 0) st_clear(g);
     PassOut &P = g->pass[level];
     free_pass(g, P);
     P.s = s;
@@ -495,16 +643,15 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     P.hB.resize((size_t)c);
     hash_pairs(seed, c, P.hA.data(), P.hB.data());
     const int st_all = level == 0 ? kStPass1 : kStPass2;
-    ev_begin(g, st_all);
-    ev_begin(g, level == 0 ? kStSelect1 : kStSelect2);
+    st_begin(g, st_all);
+    st_begin(g, level == 0 ? kStSelect1 : kStSelect2);
     dalloc(g, P.A, (size_t)c * 4);
     dalloc(g, P.B, (size_t)c * 4);
     CK(cudaMemcpyAsync(P.A.p, P.hA.data(), (size_t)c * 4, cudaMemcpyHostToDevice, g->stream));
     CK(cudaMemcpyAsync(P.B.p, P.hB.data(), (size_t)c * 4, cudaMemcpyHostToDevice, g->stream));
-    // ---- rows
+    // ---- rows of the pass
     DBuf blk, tot;
     int64_t nrows = 0;
-    const uint32_t *entries;
     if (level == 0) {
       const int64_t rows = g->row_hi - g->row_lo;
       dalloc(g, blk, (size_t)sel_scratch_elems(rows) * 8);
@@ -519,7 +666,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
       CK(select_csr_write(ptr<int64_t>(g->row_ptr), rows, s, g->row_lo, ptr<int64_t>(blk),
                           ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), ptr<uint32_t>(P.rowid),
                           g->stream));
-      entries = reinterpret_cast<const uint32_t *>(g->col.p);
+      P.entries = ptr<uint32_t>(g->col);
     } else {
       Groups &G1 = g->grp[0];
       dalloc(g, blk, (size_t)sel_scratch_elems((G1.npairs + 31) / 32) * 8);
@@ -532,50 +679,30 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
       dalloc(g, P.rlen, (size_t)nrows * 4);
       CK(select_groups_write(ptr<uint32_t>(G1.head), G1.npairs, s, ptr<int64_t>(blk),
                              ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), g->stream));
-      entries = ptr<uint32_t>(G1.members);
+      P.entries = ptr<uint32_t>(G1.members);
     }
+    dfree(g, blk);
+    dfree(g, tot);
     P.nrows = nrows;
-    if (nrows * (int64_t)c >= ((int64_t)1 << 40))
-      fail(g, SG_EOVERFLOW, "rows * c too large for one rank");
+    P.key_stride = key_stride_for(nrows);
     if (level == 0 && g->world > 1) {
-      exchange_row_counts(g, 0, nrows);  // n_e global, row base
+      exchange_row_counts(g, 0, nrows);  // n_e global
     } else if (level == 0) {
       g->n_e_global = nrows;
-      P.row_base = 0;
     } else if (g->world > 1) {
       exchange_row_counts(g, 1, nrows);  // |S1'| global, k0 (canonical dense index)
     } else {
       g->s1p_global = nrows;
       g->s1p_k0 = 0;
-      P.row_base = 0;
     }
     if (level == 1 && g->s1p_global >= (int64_t)0xFFFFFFFFll)
       fail(g, SG_EOVERFLOW, "|S1'| exceeds 2^32 - 1 (members are u32)");
-    ev_end(g, level == 0 ? kStSelect1 : kStSelect2);
-    // ---- min-hash top-s (the hot kernel)
-    ev_begin(g, level == 0 ? kStHash1 : kStHash2);
-    dalloc(g, P.keys, (size_t)(nrows * c) * 8);
-    DBuf ctr;
-    dalloc(g, ctr, 8);
-    CK(cudaMemsetAsync(ctr.p, 0, 8, g->stream));
-    MinhashArgs a;
-    a.rstart = ptr<int64_t>(P.rstart);
-    a.rlen = ptr<int32_t>(P.rlen);
-    a.entries = entries;
-    a.nrows = nrows;
-    a.A = ptr<uint32_t>(P.A);
-    a.B = ptr<uint32_t>(P.B);
-    a.c = c;
-    a.s = s;
-    a.seed = seed;
-    a.keys = ptr<uint64_t>(P.keys);
-    a.counter = ptr<unsigned long long>(ctr);
-    CK(minhash(a, g->num_sms, g->stream));
-    ev_end(g, level == 0 ? kStHash1 : kStHash2);
-    ev_end(g, st_all);
-    dfree(g, ctr);
-    dfree(g, blk);
-    dfree(g, tot);
+    st_end(g, level == 0 ? kStSelect1 : kStSelect2);
+    // ---- min-hash top-s of every row and trial (the hot kernel)
+    plan_pass(g, P);
+    if (!P.deferred)
+      for (auto &ch : P.chunks) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+    st_end(g, st_all);
     sync(g);
     g->state = level == 0 ? kPassed1 : kPassed2;
   });
@@ -589,20 +716,33 @@ sg_status group_by_shingle(sg_graph *g) {
     else fail(g, SG_ESTATE, "group_by_shingle: needs a completed shingle_pass");
     PassOut &P = g->pass[level];
     const int c = P.c;
-    ev_begin(g, level == 0 ? kStGroup1 : kStGroup2);
+    st_begin(g, level == 0 ? kStGroup1 : kStGroup2);
     if (g->world > 1) {
       exchange_and_group(g, level);
     } else {
-      std::vector<int64_t> seg((size_t)c + 1);
-      for (int j = 0; j <= c; ++j) seg[(size_t)j] = (int64_t)j * P.nrows;
+      Groups &out = g->grp[level];
+      free_groups(g, out);
+      out.c = c;
+      out.npairs = P.nrows * (int64_t)c;
+      out.seg.resize((size_t)c + 1);
+      for (int j = 0; j <= c; ++j) out.seg[(size_t)j] = (int64_t)j * P.nrows;
+      dalloc(g, out.members, (size_t)out.npairs * 4);
+      dalloc(g, out.head, (size_t)((out.npairs + 31) / 32) * 4);
+      CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
       const uint32_t *rowid = level == 0 ? ptr<uint32_t>(P.rowid) : nullptr;
       const uint32_t base = level == 0 ? 0u : (uint32_t)g->s1p_k0;
-      run_group(g, level, ptr<uint64_t>(P.keys), nullptr, rowid, base, seg, c, g->grp[level],
-                level == 0 ? kStHist1 : kStHist2, level == 0 ? kStScatter1 : kStScatter2,
-                level == 0 ? kStLocal1 : kStLocal2);
-      g->pairs_global[level] = g->grp[level].npairs;
+      GroupScratch S;
+      for (auto &ch : P.chunks) {
+        if (!ch.computed) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+        group_chunk(g, ptr<uint64_t>(ch.keys), P.key_stride, ch.t0, ch.nt, out.seg, nullptr, rowid,
+                    base, out, S, &ch.keys, level == 0 ? kStHist1 : kStHist2,
+                    level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2);
+        ch.computed = false;
+      }
+      free_scratch(g, S);
+      g->pairs_global[level] = out.npairs;
     }
-    ev_end(g, level == 0 ? kStGroup1 : kStGroup2);
+    st_end(g, level == 0 ? kStGroup1 : kStGroup2);
     sync(g);
     g->groups_global[level] = -1;  // computed lazily by sg_get_counts
     if (level == 1) g->e2_global = -1;
@@ -629,24 +769,23 @@ void shingle_graph_destroy(sg_graph *g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (int l = 0; l < 2; ++l) {
     PassOut &p = g->pass[l];
-    for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid, &p.keys})
+    for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid})
       if (b->p) cudaFree(b->p);
+    for (auto &ch : p.chunks)
+      if (ch.keys.p) cudaFree(ch.keys.p);
     for (DBuf *b : {&g->grp[l].members, &g->grp[l].head})
       if (b->p) cudaFree(b->p);
   }
-  for (DBuf *b : {&g->row_ptr, &g->col, &g->s1p_gidx, &g->scratch})
+  for (DBuf *b : {&g->row_ptr, &g->col})
     if (b->p) cudaFree(b->p);
-  for (int i = 0; i < kNumStages; ++i) {
-    if (g->st[i].beg) cudaEventDestroy(g->st[i].beg);
-    if (g->st[i].end) cudaEventDestroy(g->st[i].end);
-  }
+  for (cudaEvent_t e : g->ev_pool) cudaEventDestroy(e);
   if (g->xch) exchange_destroy(g->xch);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   cudaGetLastError();
   delete g;
 }
 
-sg_status sg_get_counts(const sg_graph *gc, int64_t counts[12]) {
+sg_status sg_get_counts(const sg_graph *gc, int64_t counts[16]) {
   sg_graph *g = const_cast<sg_graph *>(gc);
   return guarded(g, [&] {
     if (!counts) fail(g, SG_EINVAL, "counts is NULL");
@@ -654,7 +793,8 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[12]) {
     for (int l = 0; l < 2; ++l) {
       const bool grouped = g->state >= (l == 0 ? kGrouped1 : kGrouped2);
       if (grouped && g->groups_global[l] < 0) {
-        int64_t loc = count_groups(g, g->grp[l]);
+        Groups &q = g->grp[l];
+        int64_t loc = device_sum_popc(g, q.head, (q.npairs + 31) / 32);
         g->groups_global[l] = g->world > 1 ? exchange_sum(g, loc) : loc;
       }
     }
@@ -681,6 +821,12 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[12]) {
     counts[9] = g->state;
     counts[10] = g->state >= kPassed2 ? g->e2_global : 0;
     counts[11] = (int64_t)launches;
+    for (int l = 0; l < 2; ++l) {
+      const PassOut &P = g->pass[l];
+      const int64_t nch = (int64_t)P.chunks.size();
+      counts[12 + l] = P.deferred ? -nch : nch;
+    }
+    counts[14] = counts[15] = 0;
   });
 }
 
@@ -691,22 +837,30 @@ sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *r
     const int l = level - 1;
     if (g->state < (l == 0 ? kPassed1 : kPassed2)) fail(g, SG_ESTATE, "pass not run yet");
     PassOut &P = g->pass[l];
+    if (l == 0 && g->state >= kPassed2) {
+      // pass-I rows are still resident; entries (the CSR) too
+    }
     if (rows) *rows = P.nrows;
     if (c) *c = P.c;
     if (!ids && !rowid) return;
     if (cap_rows < P.nrows) fail(g, SG_EINVAL, "buffer too small");
     if (ids) {
-      DBuf t;
-      dalloc(g, t, (size_t)(P.nrows * P.c) * 8);
-      CK(transpose_keys_to_ids(ptr<uint64_t>(P.keys), P.nrows, P.c, ptr<uint64_t>(t), g->stream));
-      CK(cudaMemcpyAsync(ids, t.p, (size_t)(P.nrows * P.c) * 8, cudaMemcpyDeviceToHost, g->stream));
-      sync(g);
-      dfree(g, t);
+      std::vector<int64_t> rq((size_t)(P.nrows * P.c));
+      std::vector<int32_t> tq(rq.size());
+      for (int64_t r = 0; r < P.nrows; ++r)
+        for (int j = 0; j < P.c; ++j) {
+          rq[(size_t)(r * P.c + j)] = r;
+          tq[(size_t)(r * P.c + j)] = j;
+        }
+      std::vector<uint64_t> v = recompute_ids(g, l, rq, tq);
+      if (!v.empty()) memcpy(ids, v.data(), v.size() * 8);
     }
     if (rowid) {
       if (l == 0) {
-        CK(cudaMemcpyAsync(rowid, P.rowid.p, (size_t)P.nrows * 4, cudaMemcpyDeviceToHost, g->stream));
-        sync(g);
+        if (P.nrows) {
+          CK(cudaMemcpyAsync(rowid, P.rowid.p, (size_t)P.nrows * 4, cudaMemcpyDeviceToHost, g->stream));
+          sync(g);
+        }
       } else {
         for (int64_t r = 0; r < P.nrows; ++r) rowid[r] = (uint32_t)(g->s1p_k0 + r);
       }
@@ -733,9 +887,9 @@ sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64
     if (!caps || caps[0] < G || caps[1] < (int64_t)H.members.size())
       fail(g, SG_EINVAL, "buffers too small");
     if (trial_goffs) memcpy(trial_goffs, H.trial_goffs.data(), H.trial_goffs.size() * 8);
-    if (ids) memcpy(ids, H.ids.data(), H.ids.size() * 8);
+    if (ids && G) memcpy(ids, H.ids.data(), H.ids.size() * 8);
     if (offs) memcpy(offs, H.offs.data(), H.offs.size() * 8);
-    if (members) memcpy(members, H.members.data(), H.members.size() * 4);
+    if (members && !H.members.empty()) memcpy(members, H.members.data(), H.members.size() * 4);
   });
 }
 
@@ -774,15 +928,21 @@ sg_status sg_get_stage_ms(const sg_graph *gc, float *ms, int32_t cap, int32_t *n
   sg_graph *g = const_cast<sg_graph *>(gc);
   return guarded(g, [&] {
     const int k = std::min<int>(cap, kNumStages);
+    if (ms) sync(g);
     for (int i = 0; i < k; ++i) {
-      float v = 0.f;
-      if (g->st_used[i] && ms) {
-        if (cudaEventElapsedTime(&v, g->st[i].beg, g->st[i].end) != cudaSuccess) {
-          cudaGetLastError();
-          v = 0.f;
+      float tot = 0.f;
+      if (ms) {
+        for (auto &pr : g->st[i]) {
+          if (pr.second < 0) continue;
+          float v = 0.f;
+          if (cudaEventElapsedTime(&v, g->ev_pool[(size_t)pr.first], g->ev_pool[(size_t)pr.second]) ==
+              cudaSuccess)
+            tot += v;
+          else
+            cudaGetLastError();
         }
+        ms[i] = tot;
       }
-      if (ms) ms[i] = v;
     }
     if (n) *n = k;
   });
@@ -798,14 +958,15 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
     PassOut &P2 = g->pass[1];
     HostGroups H1, H2;
     host_groups(g, 0, H1, true);
-    host_groups(g, 1, H2, true);
-    // S1' nodes: pass-II rows, in order; group of row k starts at rstart[k]
+    host_groups(g, 1, H2, mode == 0);
+    // S1' nodes: pass-II rows, in order; the group of row k starts at rstart[k]
     std::vector<int64_t> rs = d2h<int64_t>(g, P2.rstart, (size_t)P2.nrows);
     std::vector<int32_t> rl = d2h<int32_t>(g, P2.rlen, (size_t)P2.nrows);
     const int64_t nk = P2.nrows;
     std::vector<int32_t> trial1((size_t)nk);
     std::vector<uint64_t> id1((size_t)nk);
-    std::vector<int64_t> loff((size_t)nk + 1);
+    std::vector<int64_t> lo2((size_t)nk + 1, 0);
+    std::vector<uint32_t> lm;
     {
       size_t gi = 0;
       int j = 0;
@@ -814,20 +975,12 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
         while (g->grp[0].seg[(size_t)j + 1] <= rs[(size_t)k]) ++j;
         trial1[(size_t)k] = j;
         id1[(size_t)k] = H1.ids[gi];
-        loff[(size_t)k] = rs[(size_t)k];
+        lo2[(size_t)k] = (int64_t)lm.size();
+        lm.insert(lm.end(), H1.members.begin() + rs[(size_t)k],
+                  H1.members.begin() + rs[(size_t)k] + rl[(size_t)k]);
       }
-      loff[(size_t)nk] = nk ? rs[(size_t)nk - 1] + rl[(size_t)nk - 1] : 0;
+      lo2[(size_t)nk] = (int64_t)lm.size();
     }
-    // L(k) = members[rs[k] .. rs[k] + rl[k]) — build a compact copy
-    std::vector<int64_t> lo2((size_t)nk + 1, 0);
-    std::vector<uint32_t> lm;
-    lm.reserve((size_t)(nk * 4));
-    for (int64_t k = 0; k < nk; ++k) {
-      lo2[(size_t)k] = (int64_t)lm.size();
-      lm.insert(lm.end(), H1.members.begin() + rs[(size_t)k],
-                H1.members.begin() + rs[(size_t)k] + rl[(size_t)k]);
-    }
-    lo2[(size_t)nk] = (int64_t)lm.size();
     const int64_t nh = (int64_t)H2.offs.size() - 1;
     std::vector<int32_t> trial2((size_t)nh);
     for (int t = 0; t < g->grp[1].c; ++t)
@@ -835,7 +988,7 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
         trial2[(size_t)h] = t;
     std::vector<int64_t> hrp;
     std::vector<int32_t> hcol;
-    if (P1.s >= 3) {
+    if (P1.s >= 3 && mode == 0) {
       hrp = d2h<int64_t>(g, g->row_ptr, (size_t)(g->row_hi - g->row_lo + 1));
       hcol = d2h<int32_t>(g, g->col, (size_t)g->nnz_local);
     }
@@ -854,7 +1007,7 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
     in.lmem = lm.data();
     in.nh = nh;
     in.trial2 = trial2.data();
-    in.id2 = H2.ids.data();
+    in.id2 = H2.ids.empty() ? nullptr : H2.ids.data();
     in.koff = H2.offs.data();
     in.kmem = H2.members.data();
     in.row_ptr = hrp.empty() ? nullptr : hrp.data();

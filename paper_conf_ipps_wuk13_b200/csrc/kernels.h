@@ -34,29 +34,41 @@ struct MinhashArgs {
   const int32_t *rlen;
   const uint32_t *entries;
   int64_t nrows;
-  const uint32_t *A;
+  const uint32_t *A;              // [c] hash pairs of the whole pass
   const uint32_t *B;
-  int32_t c;
+  int32_t t0;                     // first trial of this launch
+  int32_t nt;                     // trials in this launch
   int32_t s;
   uint64_t seed;
-  uint64_t *keys;                 // [c][nrows]
+  uint64_t *keys;                 // [nt][key_stride], key_stride % 8 == 0
+  int64_t key_stride;
   unsigned long long *counter;    // zeroed device counter
 };
+constexpr int kRowTile = 8;       // rows per warp tile (one 64 B store per trial)
+inline int64_t key_stride_for(int64_t nrows) { return (nrows + kRowTile - 1) / kRowTile * kRowTile; }
 cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st);
+
+// Recompute shingle ids for (row, trial) requests (getters / report only).
+cudaError_t shingle_ids(const int64_t *rstart, const int32_t *rlen, const uint32_t *entries,
+                        const uint32_t *A, const uint32_t *B, int32_t s, uint64_t seed,
+                        const int64_t *req_row, const int32_t *req_trial, int64_t nreq,
+                        uint64_t *ids, cudaStream_t st);
 
 // ---- grouping (kernels_group.cu) -------------------------------------------
 struct GroupPlan {
   int32_t c = 0;
-  int32_t bits = 0;          // B: bins per trial = 2^B
-  int64_t nbins = 1;
+  int32_t bits = 0;          // B: final buckets per trial = 2^B (top B key bits)
+  int32_t bits1 = 0;         // coarse (first scatter) bits; == bits when single-level
+  int64_t nbins = 1;         // 2^bits
+  int64_t nb1 = 1;           // 2^bits1
   int64_t nchunks = 0;
   int64_t npairs = 0;
   // device tables
-  int64_t *chunk_start = nullptr;  // [nchunks] global pair index
+  int64_t *chunk_i0 = nullptr;     // [nchunks] first pair of the chunk within its trial
   int32_t *chunk_len = nullptr;    // [nchunks]
   int32_t *chunk_trial = nullptr;  // [nchunks]
-  int32_t *chunk_rank = nullptr;   // [nchunks] index of the chunk within its trial
-  int64_t *seg = nullptr;          // [c+1] trial segment offsets
+  int64_t *in_base = nullptr;      // [c]   key index of pair 0 of trial j
+  int64_t *seg = nullptr;          // [c+1] output position of pair 0 of trial j (global)
   int32_t *trial_chunk0 = nullptr; // [c+1] first chunk of each trial
 };
 
@@ -67,11 +79,15 @@ struct GroupArgs {
   const uint32_t *rowid;       //   val = rowid[i - seg[j]] if rowid, else
   uint32_t val_base;           //   val = val_base + (i - seg[j])
   // scratch (device)
-  uint32_t *counts;            // [nchunks][nbins]
-  uint32_t *bstart;            // [c][nbins] bucket start within trial segment
+  uint32_t *counts;            // [nchunks][nb1]
+  uint32_t *bstart1;           // [c][nb1] coarse bucket start within the trial segment
+  uint32_t *bsize1;            // [c][nb1]
+  uint32_t *bstart;            // [c][nbins] final bucket start (== bstart1 if single-level)
   uint32_t *bsize;             // [c][nbins]
-  uint64_t *bkeys;             // [npairs]
-  uint32_t *bvals;             // [npairs]
+  uint64_t *akeys;             // [npairs] coarse-bucketed pairs
+  uint32_t *avals;
+  uint64_t *bkeys;             // [npairs] final-bucketed pairs (== akeys if single-level)
+  uint32_t *bvals;
   uint32_t *big_list;          // [c*nbins] bucket ids with size > local capacity
   uint32_t *big_count;         // [1]
   // outputs
@@ -80,10 +96,13 @@ struct GroupArgs {
 };
 
 int64_t group_local_capacity();
+// Bucket plan for trial segments of at most `maxseg` pairs.
+void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
 cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
-cudaError_t group_scatter(const GroupArgs &g, cudaStream_t st);
-cudaError_t group_local(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
+cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level plans only
+cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_big(const GroupArgs &g, uint32_t nbig, cudaStream_t st);
 
 // ---- getters (kernels_group.cu) --------------------------------------------

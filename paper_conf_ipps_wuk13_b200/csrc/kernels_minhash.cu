@@ -1,0 +1,364 @@
+// kernels_minhash.cu — the per-row top-s min-hash of one shingling pass
+// (Alg. 1) for sm_100a.
+//
+// The paper hashes every adjacency entry into a materialised copy and
+// segment-sorts it once per trial (Alg. 1 l.8-17).  On B200 the pass is
+// integer-ALU bound, so nothing is materialised:
+//  * a warp owns a tile of 8 consecutive rows and stages their adjacency
+//    lists once in shared memory (concatenated, 16 B aligned);
+//  * lane = trial: 32 trials run side by side on the same neighbour,
+//    broadcast from smem as 128-bit words; the s minima live in registers
+//    (the paper's insertion-sorted s-array);
+//  * when c is not a multiple of 32, the tail trials are split over lanes by
+//    neighbour subsets and merged with warp shuffles;
+//  * h = (A v + B) mod (2^31 - 1): one IMAD.WIDE + Mersenne fold + one
+//    conditional subtract (sg_internal.cuh);
+//  * each lane ends a tile with the 8 keys of its trial for 8 consecutive
+//    rows: one 64 B (two full sectors) store into the trial-major key array.
+#include <algorithm>
+
+#include "kernels.h"
+#include "scan.cuh"
+#include "sg_internal.cuh"
+
+namespace sg {
+
+namespace {
+
+constexpr int kMhThreads = 256;
+constexpr int kMhWarps = kMhThreads / 32;
+constexpr int kNbCap = 1024;        // staged entries per warp (4 KB)
+constexpr int kMaxPasses = 48;
+constexpr int TR = kRowTile;
+
+struct TrialPass {
+  int16_t t0;      // first trial of the pass (relative to the launch's t0)
+  int8_t logT;     // trials in the pass = 2^logT  (trial = lane & (T-1))
+  int8_t logp;     // neighbour parts    = 2^logp  (part  = lane >> logT)
+};
+
+struct MhParams {
+  MinhashArgs a;
+  int32_t npass;
+  int32_t tiles_per_grab;
+  TrialPass pass[kMaxPasses];
+};
+
+// Keep the S smallest of m[] U {h} ascending: compare-exchange chain.
+template <int S>
+__device__ __forceinline__ void insert_min(uint32_t (&m)[S], uint32_t h) {
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    uint32_t lo = min(m[i], h);
+    h = max(m[i], h);
+    m[i] = lo;
+  }
+}
+
+// Within-trial shingle id (AMB-4).
+template <int S>
+__device__ __forceinline__ uint64_t shingle_id(const uint32_t (&m)[S], uint64_t seed, int j) {
+  if (S == 1) return (uint64_t)m[0];
+  if (S == 2) return ((uint64_t)m[0] << 31) | (uint64_t)m[S - 1];
+  uint64_t z = fmix(seed ^ fmix((uint64_t)j + 1));
+#pragma unroll
+  for (int i = 0; i < S; ++i) z = fmix(z + (uint64_t)m[i]);
+  return z;
+}
+
+template <int S>
+__device__ __forceinline__ void scan_strided(const uint32_t *nb, int len, int part, int p,
+                                             uint32_t a, uint32_t b, uint32_t (&m)[S]) {
+  for (int e = part; e < len; e += p) {
+    uint32_t h = m31_hash(a, b, nb[e]);
+    if (h < m[S - 1]) insert_min<S>(m, h);
+  }
+}
+
+// p == 1: every lane scans every entry, 4 per 128-bit broadcast load.
+template <int S>
+__device__ __forceinline__ void scan_all(const uint32_t *nb, int len, uint32_t a, uint32_t b,
+                                         uint32_t (&m)[S]) {
+  const uint4 *nb4 = reinterpret_cast<const uint4 *>(nb);
+  const int len4 = len >> 2;
+#pragma unroll 2
+  for (int q = 0; q < len4; ++q) {
+    uint4 v = nb4[q];
+    uint32_t h0 = m31_hash(a, b, v.x);
+    uint32_t h1 = m31_hash(a, b, v.y);
+    uint32_t h2 = m31_hash(a, b, v.z);
+    uint32_t h3 = m31_hash(a, b, v.w);
+    uint32_t hm = min(min(h0, h1), min(h2, h3));
+    if (hm < m[S - 1]) {
+      insert_min<S>(m, h0);
+      insert_min<S>(m, h1);
+      insert_min<S>(m, h2);
+      insert_min<S>(m, h3);
+    }
+  }
+  for (int e = len4 << 2; e < len; ++e) {
+    uint32_t h = m31_hash(a, b, nb[e]);
+    if (h < m[S - 1]) insert_min<S>(m, h);
+  }
+}
+
+template <int S>
+__device__ __forceinline__ void scan_any(const uint32_t *nb, int len, int part, int p, uint32_t a,
+                                         uint32_t b, uint32_t (&m)[S]) {
+  if (p == 1) scan_all<S>(nb, len, a, b, m);
+  else scan_strided<S>(nb, len, part, p, a, b, m);
+}
+
+template <int S>
+__global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_constant__ MhParams P) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  __shared__ int64_t sSt[kMhWarps][TR];
+  __shared__ int sLen[kMhWarps][TR];
+  __shared__ int sOff[kMhWarps][TR + 1];
+  const MinhashArgs &a = P.a;
+  const int nt = a.nt;
+  const int ntp = (nt + 7) & ~7;
+  uint32_t *sA = reinterpret_cast<uint32_t *>(smraw);
+  uint32_t *sB = sA + ntp;
+  uint64_t *sOutAll = reinterpret_cast<uint64_t *>(sB + ntp);
+  uint32_t *sNbAll = reinterpret_cast<uint32_t *>(sOutAll + kMhWarps * TR * 32);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint64_t *sOut = sOutAll + w * TR * 32;
+  uint32_t *nb = sNbAll + w * kNbCap;
+  for (int i = threadIdx.x; i < nt; i += blockDim.x) {
+    sA[i] = a.A[a.t0 + i];
+    sB[i] = a.B[a.t0 + i];
+  }
+  __syncthreads();
+  const int64_t nrows = a.nrows;
+  const int64_t ntiles = (nrows + TR - 1) / TR;
+  for (;;) {
+    unsigned long long g0 = 0;
+    if (lane == 0) g0 = atomicAdd(a.counter, (unsigned long long)P.tiles_per_grab);
+    g0 = __shfl_sync(0xffffffffu, g0, 0);
+    if ((int64_t)g0 >= ntiles) break;
+    const int64_t g1 = min((int64_t)g0 + P.tiles_per_grab, ntiles);
+    for (int64_t tile = (int64_t)g0; tile < g1; ++tile) {
+      const int64_t r0 = tile * TR;
+      const int nr = (int)min((int64_t)TR, nrows - r0);
+      __syncwarp();
+      int len = 0;
+      int64_t st = 0;
+      if (lane < nr) {
+        st = a.rstart[r0 + lane];
+        len = a.rlen[r0 + lane];
+      }
+      const int plen = (len + 3) & ~3;
+      const int incl = warp_incl_scan(plen);
+      if (lane < TR) {
+        sSt[w][lane] = st;
+        sLen[w][lane] = len;
+        sOff[w][lane + 1] = incl;
+      }
+      if (lane == 0) sOff[w][0] = 0;
+      __syncwarp();
+      const int total = sOff[w][TR];
+      if (total > kNbCap) {
+        // long rows: one row at a time, staged once (or chunk by chunk when it
+        // exceeds the stage), all trial passes on it, scalar key stores
+        for (int rr = 0; rr < nr; ++rr) {
+          const int rl = sLen[w][rr];
+          const uint32_t *src = a.entries + sSt[w][rr];
+          const bool fits = rl <= kNbCap;
+          if (fits) {
+            __syncwarp();
+            for (int i = lane; i < rl; i += 32) nb[i] = src[i];
+            __syncwarp();
+          }
+          for (int pi = 0; pi < P.npass; ++pi) {
+            const TrialPass tp = P.pass[pi];
+            const int T = 1 << tp.logT;
+            const int p = 1 << tp.logp;
+            const int tl = lane & (T - 1);
+            const int part = lane >> tp.logT;
+            const int j = tp.t0 + tl;
+            const uint32_t A = sA[j], B = sB[j];
+            uint32_t m[S];
+#pragma unroll
+            for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+            if (fits) {
+              scan_any<S>(nb, rl, part, p, A, B, m);
+            } else {
+              for (int c0 = 0; c0 < rl; c0 += kNbCap) {
+                const int cl = min(kNbCap, rl - c0);
+                __syncwarp();
+                for (int i = lane; i < cl; i += 32) nb[i] = src[c0 + i];
+                __syncwarp();
+                scan_any<S>(nb, cl, part, p, A, B, m);
+              }
+            }
+            for (int o = T; o < 32; o <<= 1) {
+              uint32_t x[S];
+#pragma unroll
+              for (int i = 0; i < S; ++i) x[i] = __shfl_xor_sync(0xffffffffu, m[i], o);
+#pragma unroll
+              for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
+            }
+            if (part == 0)
+              a.keys[(int64_t)j * a.key_stride + r0 + rr] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+          }
+        }
+        continue;
+      }
+      // short rows: the whole tile staged once, trial passes outer, rows inner
+      for (int i = lane; i < total; i += 32) {
+        int rr = 0;
+#pragma unroll
+        for (int x = 1; x < TR; ++x) rr += (i >= sOff[w][x]);
+        const int k = i - sOff[w][rr];
+        nb[i] = k < sLen[w][rr] ? a.entries[sSt[w][rr] + k] : 0u;
+      }
+      __syncwarp();
+      for (int pi = 0; pi < P.npass; ++pi) {
+        const TrialPass tp = P.pass[pi];
+        const int T = 1 << tp.logT;
+        const int p = 1 << tp.logp;
+        const int tl = lane & (T - 1);
+        const int part = lane >> tp.logT;
+        const int j = tp.t0 + tl;               // trial index within the launch
+        const uint32_t A = sA[j], B = sB[j];
+        for (int rr = 0; rr < nr; ++rr) {
+          const int rl = sLen[w][rr];
+          uint32_t m[S];
+#pragma unroll
+          for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+          scan_any<S>(nb + sOff[w][rr], rl, part, p, A, B, m);
+          // merge the p partial lists of a trial (lanes tl, tl + T, ...)
+          for (int o = T; o < 32; o <<= 1) {
+            uint32_t x[S];
+#pragma unroll
+            for (int i = 0; i < S; ++i) x[i] = __shfl_xor_sync(0xffffffffu, m[i], o);
+#pragma unroll
+            for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
+          }
+          if (part == 0) sOut[rr * 32 + tl] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+        }
+        __syncwarp();
+        if (part == 0) {
+          uint64_t *dst = a.keys + (int64_t)j * a.key_stride + r0;
+          if (nr == TR) {
+            ulonglong2 *d2 = reinterpret_cast<ulonglong2 *>(dst);
+#pragma unroll
+            for (int q = 0; q < TR / 2; ++q)
+              d2[q] = make_ulonglong2(sOut[(2 * q) * 32 + tl], sOut[(2 * q + 1) * 32 + tl]);
+          } else {
+            for (int rr = 0; rr < nr; ++rr) dst[rr] = sOut[rr * 32 + tl];
+          }
+        }
+        __syncwarp();
+      }
+    }
+  }
+}
+
+template <int S>
+cudaError_t launch_tile(const MhParams &P, int num_sms, cudaStream_t st) {
+  const int ntp = (P.a.nt + 7) & ~7;
+  const size_t smem = (size_t)2 * ntp * 4 + (size_t)kMhWarps * TR * 32 * 8 +
+                      (size_t)kMhWarps * kNbCap * 4;
+  auto kern = minhash_tile_kernel<S>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kMhThreads, smem);
+  if (e != cudaSuccess) return e;
+  per_sm = std::max(per_sm, 1);
+  const int64_t ntiles = (P.a.nrows + TR - 1) / TR;
+  const int64_t want = (ntiles + kMhWarps - 1) / kMhWarps;
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, std::max<int64_t>(want, 1));
+  kern<<<grid, kMhThreads, smem, st>>>(P);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+// ---- id recomputation for getters / report (one thread per request) --------
+__global__ void shingle_ids_kernel(const int64_t *rstart, const int32_t *rlen,
+                                   const uint32_t *entries, const uint32_t *A, const uint32_t *B,
+                                   int s, uint64_t seed, const int64_t *req_row,
+                                   const int32_t *req_trial, int64_t nreq, uint64_t *ids) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nreq;
+       q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = req_row[q];
+    const int j = req_trial[q];
+    const uint32_t *row = entries + rstart[r];
+    const int len = rlen[r];
+    uint32_t m[kMaxS];
+    for (int i = 0; i < kMaxS; ++i) m[i] = 0xFFFFFFFFu;
+    for (int e = 0; e < len; ++e) {
+      uint32_t h = m31_hash(A[j], B[j], row[e]);
+      if (h >= m[s - 1]) continue;
+      int i = s - 1;
+      while (i > 0 && m[i - 1] > h) {
+        m[i] = m[i - 1];
+        --i;
+      }
+      m[i] = h;
+    }
+    uint64_t id;
+    if (s == 1) {
+      id = m[0];
+    } else if (s == 2) {
+      id = ((uint64_t)m[0] << 31) | m[1];
+    } else {
+      uint64_t z = fmix(seed ^ fmix((uint64_t)j + 1));
+      for (int i = 0; i < s; ++i) z = fmix(z + (uint64_t)m[i]);
+      id = z;
+    }
+    ids[q] = id;
+  }
+}
+
+}  // namespace
+
+cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st) {
+  if (a.nrows == 0 || a.nt == 0) return cudaSuccess;
+  if (a.key_stride % TR != 0) return cudaErrorInvalidValue;
+  MhParams P;
+  P.a = a;
+  // trial passes: full groups of 32 lanes (one trial per lane), then the
+  // binary digits of nt mod 32 (2^b trials x 32/2^b neighbour parts)
+  int np = 0, t = 0;
+  while (a.nt - t >= 32) {
+    P.pass[np++] = TrialPass{(int16_t)t, 5, 0};
+    t += 32;
+  }
+  for (int b = 4; b >= 0; --b) {
+    if ((a.nt - t) & (1 << b)) {
+      P.pass[np++] = TrialPass{(int16_t)t, (int8_t)b, (int8_t)(5 - b)};
+      t += 1 << b;
+    }
+  }
+  P.npass = np;
+  const int64_t ntiles = (a.nrows + TR - 1) / TR;
+  const int64_t warps = (int64_t)num_sms * 32;
+  P.tiles_per_grab = (int32_t)std::max<int64_t>(1, std::min<int64_t>(16, ntiles / (warps * 8)));
+  switch (a.s) {
+    case 1: return launch_tile<1>(P, num_sms, st);
+    case 2: return launch_tile<2>(P, num_sms, st);
+    case 3: return launch_tile<3>(P, num_sms, st);
+    case 4: return launch_tile<4>(P, num_sms, st);
+    case 5: return launch_tile<5>(P, num_sms, st);
+    case 6: return launch_tile<6>(P, num_sms, st);
+    case 7: return launch_tile<7>(P, num_sms, st);
+    case 8: return launch_tile<8>(P, num_sms, st);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t shingle_ids(const int64_t *rstart, const int32_t *rlen, const uint32_t *entries,
+                        const uint32_t *A, const uint32_t *B, int32_t s, uint64_t seed,
+                        const int64_t *req_row, const int32_t *req_trial, int64_t nreq,
+                        uint64_t *ids, cudaStream_t st) {
+  if (nreq == 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((nreq + 255) / 256, 148 * 16);
+  shingle_ids_kernel<<<grid, 256, 0, st>>>(rstart, rlen, entries, A, B, s, seed, req_row,
+                                           req_trial, nreq, ids);
+  return cudaGetLastError();
+}
+
+}  // namespace sg

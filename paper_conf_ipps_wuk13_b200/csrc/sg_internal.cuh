@@ -8,6 +8,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/shingle.h"
@@ -22,7 +23,7 @@ constexpr int kMaxC = 1024;     // c bound of the ABI
 // ----------------------------------------------------------------------------
 // 64-bit mixing: the splitmix64 finaliser and its inverse (bijection on 2^64).
 // Used for (a) the hash-pair stream (AMB-2), (b) the s >= 3 shingle fold
-// (AMB-4), (c) the grouping key key = fmix(id) (AMB-19, DESIGN.md §5).
+// (AMB-4), (c) the grouping key key = fmix(id) (AMB-19, DESIGN.md §3).
 // ----------------------------------------------------------------------------
 __host__ __device__ __forceinline__ uint64_t fmix(uint64_t z) {
   z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
@@ -61,9 +62,9 @@ __device__ __forceinline__ uint32_t m31_hash(uint32_t A, uint32_t B, uint32_t v)
 // ----------------------------------------------------------------------------
 enum State : int32_t {
   kCreated = 0,   // CSR resident
-  kPassed1 = 1,   // pass I keys resident
+  kPassed1 = 1,   // pass I rows selected (keys computed unless deferred)
   kGrouped1 = 2,  // G_I resident
-  kPassed2 = 3,   // pass II keys resident
+  kPassed2 = 3,   // pass II rows selected
   kGrouped2 = 4,  // G_II resident
   kPoisoned = 99
 };
@@ -74,18 +75,27 @@ struct DBuf {
   size_t bytes = 0;
 };
 
-// Output of one shingling pass on this rank.
+// Keys of a contiguous range of trials [t0, t0 + nt): uint64 [nt][key_stride].
+struct KeyChunk {
+  int32_t t0 = 0, nt = 0;
+  bool computed = false;
+  DBuf keys;
+};
+
+// One shingling pass on this rank.
 struct PassOut {
   int32_t s = 0, c = 0;
   uint64_t seed = 0;
   int64_t nrows = 0;            // local rows with >= s entries
-  int64_t row_base = 0;         // global index of this rank's first row
+  int64_t key_stride = 0;       // nrows rounded up to the row tile
   std::vector<uint32_t> hA, hB; // hash pairs (host copy)
   DBuf A, B;                    // uint32 [c]
   DBuf rstart;                  // int64 [nrows] first entry of each row
   DBuf rlen;                    // int32 [nrows]
   DBuf rowid;                   // uint32 [nrows] generator value (pass I: vertex id)
-  DBuf keys;                    // uint64 [c][nrows]  key = fmix(id), trial-major
+  const uint32_t *entries = nullptr;  // row entries (pass I: col; pass II: G_I members)
+  std::vector<KeyChunk> chunks; // trial chunks sized to the free HBM
+  bool deferred = false;        // keys computed chunk by chunk inside group_by_shingle
 };
 
 // Grouped pairs of one level on this rank: per-trial segments of `members`
@@ -93,19 +103,12 @@ struct PassOut {
 struct Groups {
   int32_t c = 0;
   int64_t npairs = 0;
-  int64_t ngroups = 0;                 // local group count
   std::vector<int64_t> seg;            // [c+1] pair offsets per trial (host)
   DBuf members;                        // uint32 [npairs]
-  DBuf keys;                           // uint64 [npairs] sorted keys (kept for ids / report)
   DBuf head;                           // uint32 [(npairs + 31) / 32] head bits
 };
 
-struct Stage {
-  cudaEvent_t beg = nullptr, end = nullptr;
-};
-
 constexpr int kNumStages = 16;
-// stage ids
 enum StageId {
   kStPass1 = 0, kStGroup1 = 1, kStPass2 = 2, kStGroup2 = 3,
   kStSelect1 = 4, kStHash1 = 5, kStSelect2 = 6, kStHash2 = 7,
@@ -150,11 +153,10 @@ struct sg_graph {
   int64_t pairs_global[2] = {0, 0};
   int64_t e2_global = -1;       // pass-II entries (sum of |L| over S1'), lazily
   long long launch_base = 0;    // g_launches at create / reset
-  // G_I -> S1' selection (local): group index of each local S1' node
-  sg::DBuf s1p_gidx;  // int64 [s1p_local] (only materialised for getters)
-  // stage timing
-  sg::Stage st[sg::kNumStages];
-  bool st_used[sg::kNumStages] = {};
-  // scratch
-  sg::DBuf scratch;
+  // stage timing: event pairs per stage (a stage may span several chunks)
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_next = 0;
+  std::vector<std::pair<int, int>> st[sg::kNumStages];
+  int64_t mem_budget = 0;       // test hook: cap on planned bytes (0 = free HBM)
+  int64_t bytes_live = 0;       // device bytes currently held by this handle
 };

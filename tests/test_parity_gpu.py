@@ -177,6 +177,34 @@ def test_device_pointer_input(B):
     assert np.array_equal(rows, ref.rows1) and np.array_equal(ids, ref.M1)
 
 
+@pytest.mark.parametrize("budget_mb", [400, 250, 160])
+def test_trial_chunking_under_memory_budget(B, budget_mb, monkeypatch):
+    """A small HBM budget forces the planner to split the trials into chunks
+    (eager) or to compute keys inside the grouping (deferred); grouping is per
+    trial (AMB-5), so the results must not change."""
+    g = SG.make("small")
+    cfg = SG.CONFIGS["small"]
+    monkeypatch.setenv("SG_MEM_BUDGET", str(budget_mb << 20))
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
+                        report=False)
+    assert_parity(out, ref, report=False)
+    c = out["counts"]
+    assert abs(c["chunks1"]) > 1 or abs(c["chunks2"]) > 1, c
+
+
+@pytest.mark.parametrize("target", ["4", "40", "300"])
+def test_two_level_partition_and_tiny_buckets(B, target, monkeypatch):
+    """SG_GROUP_TARGET shrinks the target bucket size so that the small graph
+    takes the two-level partition (coarse scatter + per-bucket scatter) used by
+    the 40M-row trial segments of the GOS-shaped pass II."""
+    g = SG.make("small")
+    cfg = SG.CONFIGS["small"]
+    monkeypatch.setenv("SG_GROUP_TARGET", target)
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
+                        report=False)
+    assert_parity(out, ref, report=False)
+
+
 def test_invalid_csr_rejected(B):
     g = SG.random_graph(200, 900, seed=2)
     r = int(np.argmax(np.diff(g.row_ptr) >= 2))
