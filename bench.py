@@ -188,7 +188,8 @@ def bench_ours(args, rank, world, local_rank):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     g, cfg = workload(args.config)
     s1, c1, seed1, s2, c2, seed2 = (cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()           # a non-default stream shared with the library
+    torch.cuda.set_stream(stream)
     dinfo = {"rank": rank, "world": world, "device": local_rank, "stream": stream.cuda_stream}
     if dist_on:
         uid = [None]

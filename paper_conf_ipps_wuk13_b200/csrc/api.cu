@@ -47,16 +47,56 @@ namespace {
 
 #define CK(call) ck(g, (call), #call)
 
-void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
-  if (b.p) {
-    cudaFreeAsync(b.p, g->stream);
-    g->bytes_live -= (int64_t)b.bytes;
-    b.p = nullptr;
-    b.bytes = 0;
+// Per-handle buffer cache: freed buffers are kept and handed out again by
+// best fit, so repeated runs (bench steps, resets) allocate nothing and the
+// stream-ordered pool does not fragment and grow.
+void cache_put(sg_graph *g, void *p, size_t bytes) {
+  g->cache.push_back({p, bytes});
+  g->bytes_cached += (int64_t)bytes;
+}
+
+void cache_release(sg_graph *g) {
+  for (auto &c : g->cache) cudaFreeAsync(c.p, g->stream);
+  g->cache.clear();
+  g->bytes_cached = 0;
+}
+
+void *cache_take(sg_graph *g, size_t bytes, size_t *got) {
+  size_t best = g->cache.size();
+  for (size_t i = 0; i < g->cache.size(); ++i) {
+    const size_t b = g->cache[i].bytes;
+    if (b >= bytes && b <= bytes + bytes / 4 + (1u << 20) &&
+        (best == g->cache.size() || b < g->cache[best].bytes))
+      best = i;
   }
+  if (best == g->cache.size()) return nullptr;
+  void *p = g->cache[best].p;
+  *got = g->cache[best].bytes;
+  g->bytes_cached -= (int64_t)*got;
+  g->cache.erase(g->cache.begin() + (long)best);
+  return p;
+}
+
+void dfree(sg_graph *g, DBuf &b);
+
+void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
+  if (b.p) dfree(g, b);
   if (bytes == 0) bytes = 16;
+  bytes = (bytes + 255) & ~(size_t)255;
+  size_t got = 0;
+  if (void *c = cache_take(g, bytes, &got)) {
+    b.p = c;
+    b.bytes = got;
+    g->bytes_live += (int64_t)got;
+    return;
+  }
   void *p = nullptr;
   cudaError_t e = cudaMallocAsync(&p, bytes, g->stream);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    cache_release(g);
+    e = cudaMallocAsync(&p, bytes, g->stream);
+  }
   if (e != cudaSuccess) {
     cudaGetLastError();
     size_t fr = 0, tot = 0;
@@ -74,7 +114,7 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
 
 void dfree(sg_graph *g, DBuf &b) {
   if (b.p) {
-    cudaFreeAsync(b.p, g->stream);
+    cache_put(g, b.p, b.bytes);
     g->bytes_live -= (int64_t)b.bytes;
   }
   b.p = nullptr;
@@ -185,8 +225,12 @@ int64_t avail_bytes(sg_graph *g) {
   uint64_t reserved = 0, used = 0;
   CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved));
   CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used));
-  int64_t a = (int64_t)fr + (int64_t)(reserved - used) - ((int64_t)1 << 30);
+  int64_t a = (int64_t)fr + (int64_t)(reserved - used) + g->bytes_cached - ((int64_t)1 << 30);
   if (g->mem_budget > 0) a = std::min<int64_t>(a, g->mem_budget - g->bytes_live);
+  if (getenv("SG_DEBUG_MEM"))
+    fprintf(stderr, "[sg] free %zu total %zu pool reserved %llu used %llu cached %lld live %lld -> avail %lld\n",
+            fr, tot, (unsigned long long)reserved, (unsigned long long)used,
+            (long long)g->bytes_cached, (long long)g->bytes_live, (long long)a);
   return a;
 }
 
@@ -293,7 +337,8 @@ void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, 
   const bool two = bits != bits1;
   const int64_t nbins = (int64_t)1 << bits;
   const int64_t nb1 = (int64_t)1 << bits1;
-  const int64_t CH = std::max<int64_t>(65536, 64 * nb1);
+  const int64_t CH = group_chunk_pairs();
+  (void)nb1;
   std::vector<int64_t> ci0, inb((size_t)nt), seg((size_t)nt + 1);
   std::vector<int32_t> clen, ctr, tc0((size_t)nt + 1);
   for (int j = 0; j < nt; ++j) {
@@ -617,8 +662,13 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
   }
   if (st != SG_OK) {
     if (g->xch) exchange_destroy(g->xch);
-    for (DBuf *b : {&g->row_ptr, &g->col})
-      if (b->p) cudaFree(b->p);
+    if (g->stream) {
+      for (DBuf *b : {&g->row_ptr, &g->col})
+        if (b->p) cudaFreeAsync(b->p, g->stream);
+      for (auto &c : g->cache) cudaFreeAsync(c.p, g->stream);
+      cudaStreamSynchronize(g->stream);
+    }
+    cudaGetLastError();
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
     return st;
   }
@@ -766,18 +816,20 @@ sg_status shingle_graph_reset(sg_graph *g) {
 void shingle_graph_destroy(sg_graph *g) {
   if (!g) return;
   cudaSetDevice(g->device);
-  if (g->stream) cudaStreamSynchronize(g->stream);
+  // stream-ordered frees back into the pool (cudaFree on pool blocks leaves
+  // them accounted as used), then let the pool return them to the device
+  auto rel = [&](void *p) {
+    if (p) cudaFreeAsync(p, g->stream);
+  };
   for (int l = 0; l < 2; ++l) {
     PassOut &p = g->pass[l];
-    for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid})
-      if (b->p) cudaFree(b->p);
-    for (auto &ch : p.chunks)
-      if (ch.keys.p) cudaFree(ch.keys.p);
-    for (DBuf *b : {&g->grp[l].members, &g->grp[l].head})
-      if (b->p) cudaFree(b->p);
+    for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) rel(b->p);
+    for (auto &ch : p.chunks) rel(ch.keys.p);
+    for (DBuf *b : {&g->grp[l].members, &g->grp[l].head}) rel(b->p);
   }
-  for (DBuf *b : {&g->row_ptr, &g->col})
-    if (b->p) cudaFree(b->p);
+  for (DBuf *b : {&g->row_ptr, &g->col}) rel(b->p);
+  for (auto &c : g->cache) rel(c.p);
+  if (g->stream) cudaStreamSynchronize(g->stream);
   for (cudaEvent_t e : g->ev_pool) cudaEventDestroy(e);
   if (g->xch) exchange_destroy(g->xch);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);

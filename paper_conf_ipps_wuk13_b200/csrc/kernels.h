@@ -96,6 +96,7 @@ struct GroupArgs {
 };
 
 int64_t group_local_capacity();
+int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 // Bucket plan for trial segments of at most `maxseg` pairs.
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);

@@ -1,19 +1,21 @@
-// kernels_group.cu — partition of <shingle, generator> pairs into per-trial
-// key buckets, the first half of the grouping "once for each random trial"
-// (AMB-5).  The second half (sort inside a bucket + RLE) is
-// kernels_local.cu.  DESIGN.md §6.2.
+// kernels_group.cu — stable partition of <shingle, generator> pairs into
+// per-trial key buckets: the first half of the grouping "once for each random
+// trial" (AMB-5).  The second half (sort inside a bucket + RLE)
+// is kernels_local.cu.  DESIGN.md §6.2.
 //
-//   1. hist     : per (trial, chunk) histogram of the top bits1 key bits;
+//   1. hist     : per (trial, 8K-pair chunk) histogram of the top bits1 bits;
 //   2. offsets  : column prefix over chunks + per-trial bucket scan;
-//   3. scatter  : one persistent CTA per SM writes (key, member) into coarse
-//                 (trial, bucket) order through shared-memory cursors.  The
-//                 fan-out is <= 1024 buckets, so the partially written
-//                 sectors all CTAs keep open (SMs x 1024 x 2 x 32 B < 10 MB)
-//                 stay in L2 and every sector reaches HBM complete;
-//   4. scatter2 : only when a trial segment is too long for 1024 buckets of
-//                 <= 8K pairs: one CTA per coarse bucket histograms it (the
-//                 re-read hits L2) and scatters it by the next key bits
-//                 (fan-out <= 64) into the final buckets.
+//   3. scatter  : persistent, two 16-warp CTAs per SM.  A chunk's keys are
+//                 staged in shared memory, split into 16 contiguous warp
+//                 segments and ranked stably (__match_any_sync + per-warp
+//                 bucket counters); every pair is then written straight to its
+//                 bucket slot.  Fan-out <= 1024 buckets and <= 296 concurrent
+//                 chunks keep the partially written sectors (~19 MB) in L2;
+//   4. scatter2 : only for very long trial segments (two-level plans): one
+//                 CTA per coarse bucket splits it stably by the next <= 6 bits.
+// Stability matters: the input of every trial is in generator order, so the
+// members of one group (equal keys) arrive in ascending order and the local
+// sort never has to sort a group by member.
 #include <algorithm>
 #include <cstdlib>
 
@@ -29,16 +31,101 @@ namespace {
 using grp::top_bits;
 
 constexpr int kGThreads = 512;
-constexpr int kSThreads = 1024;      // scatter: one persistent CTA per SM
-constexpr int kItems = 8;            // ILP batch per thread
-constexpr int kMaxSingleBits = 10;   // single-level fan-out bound
+constexpr int kSThreads = 512;       // 16 warps
+constexpr int kWarps = kSThreads / 32;
+constexpr int kChunk = 8192;         // pairs per scatter chunk (== hist chunk)
+constexpr int kPerLane = kChunk / kSThreads;   // 16
+constexpr int kMaxSingleBits = 10;   // single-level fan-out bound (<= 1024 buckets)
 constexpr int kCoarseBits = 9;       // two-level: first fan-out
-constexpr int kMaxBits = 14;         // final buckets per trial <= 16384
+constexpr int kMaxBits = 15;         // final buckets per trial <= 32768
+constexpr int kMaxNb1 = 1 << kMaxSingleBits;
+constexpr int kMaxNb2 = 1 << (kMaxBits - kCoarseBits);
 
 __device__ __forceinline__ uint32_t val_at(const GroupArgs &g, int64_t in_idx, int64_t i) {
   if (g.vals) return g.vals[in_idx];
   if (g.rowid) return g.rowid[i];
   return g.val_base + (uint32_t)i;
+}
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// ---- stable multi-split of the len <= kChunk keys staged in sK ---------------
+// Warp w owns the contiguous elements [w*512, w*512 + 512).  bin_of(k) in
+// [0, nb), nb <= 1024; cnt is uint16 [kWarps][nb]; sbst receives the bucket
+// starts within the chunk; emit(e, p, b) gets each element's chunk-relative
+// stable position p (bucket-major, input order inside a bucket).
+template <typename BIN, typename EMIT>
+__device__ __forceinline__ void stable_split(const uint64_t *sK, int len, int nb, BIN bin_of,
+                                             uint16_t *cnt, uint32_t *sbst, int64_t *ws,
+                                             EMIT emit) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint32_t lt = lanemask_lt();
+  uint16_t *my = cnt + w * nb;
+  for (int b = lane; b < nb; b += 32) my[b] = 0;
+  __syncwarp();
+  uint32_t pr[kPerLane];
+#pragma unroll
+  for (int u = 0; u < kPerLane; ++u) {
+    const int e = w * (kPerLane * 32) + u * 32 + lane;
+    const bool valid = e < len;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    pr[u] = 0;
+    if (valid) {
+      const uint32_t b = bin_of(sK[e]);
+      pr[u] = __match_any_sync(vm, b);
+      if ((pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
+    }
+  }
+  __syncthreads();
+  {
+    // per bucket: exclusive prefix over the warps; bucket start = exclusive
+    // prefix over the buckets (thread t owns buckets [t*per, t*per + per))
+    const int per = (nb + blockDim.x - 1) / blockDim.x;   // <= 2
+    uint32_t tot[2] = {0, 0};
+    for (int y = 0; y < per; ++y) {
+      const int b = threadIdx.x * per + y;
+      if (b < nb) {
+        uint32_t run = 0;
+        for (int x = 0; x < kWarps; ++x) {
+          const uint32_t c = cnt[x * nb + b];
+          cnt[x * nb + b] = (uint16_t)run;
+          run += c;
+        }
+        tot[y] = run;
+      }
+    }
+    int64_t all;
+    int64_t ex = block_excl_scan<int64_t>((int64_t)tot[0] + tot[1], ws, &all);
+    for (int y = 0; y < per; ++y) {
+      const int b = threadIdx.x * per + y;
+      if (b < nb) {
+        sbst[b] = (uint32_t)ex;
+        for (int x = 0; x < kWarps; ++x) cnt[x * nb + b] += (uint16_t)ex;
+      }
+      ex += tot[y];
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int u = 0; u < kPerLane; ++u) {
+    const int e = w * (kPerLane * 32) + u * 32 + lane;
+    const bool valid = e < len;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    if (valid) {
+      const uint32_t b = bin_of(sK[e]);
+      const uint32_t rank = __popc(pr[u] & lt);
+      const uint32_t base = my[b];
+      __syncwarp(vm);
+      if (rank == 0) my[b] = (uint16_t)(base + __popc(pr[u]));
+      __syncwarp(vm);
+      emit(e, (int)(base + rank), b);
+    }
+  }
+  __syncthreads();
 }
 
 // ---- 1. histogram -----------------------------------------------------------
@@ -52,17 +139,15 @@ __global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__
   const int j = g.plan.chunk_trial[k];
   const uint64_t *__restrict__ keys = g.keys + g.plan.in_base[j] + g.plan.chunk_i0[k];
   const int len = g.plan.chunk_len[k];
-  for (int base = threadIdx.x; base < len; base += blockDim.x * kItems) {
-    uint64_t kk[kItems];
+  uint64_t kk[kChunk / kGThreads];
 #pragma unroll
-    for (int u = 0; u < kItems; ++u) {
-      const int i = base + u * blockDim.x;
-      kk[u] = i < len ? keys[i] : 0;
-    }
-#pragma unroll
-    for (int u = 0; u < kItems; ++u)
-      if (base + u * (int)blockDim.x < len) atomicAdd(&hist[top_bits(kk[u], bits)], 1u);
+  for (int u = 0; u < kChunk / kGThreads; ++u) {
+    const int i = threadIdx.x + u * kGThreads;
+    kk[u] = i < len ? keys[i] : 0;
   }
+#pragma unroll
+  for (int u = 0; u < kChunk / kGThreads; ++u)
+    if (threadIdx.x + u * kGThreads < len) atomicAdd(&hist[top_bits(kk[u], bits)], 1u);
   __syncthreads();
   uint32_t *out = g.counts + k * nb;
   for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) out[i] = hist[i];
@@ -104,50 +189,65 @@ __global__ void binscan_kernel(const __grid_constant__ GroupArgs g) {
   }
 }
 
-// ---- 3. coarse scatter (persistent) -------------------------------------------
-__global__ void __launch_bounds__(kSThreads, 1) scatter_kernel(const __grid_constant__ GroupArgs g) {
-  extern __shared__ uint32_t cur[];
-  const int64_t nb = g.plan.nb1;
+// ---- 3. stable coarse scatter (persistent, 2 CTAs / SM) -----------------------
+struct ScatterSmem {
+  uint64_t K[kChunk];
+  uint16_t cnt[kWarps * kMaxNb1];
+  uint32_t sbst[kMaxNb1];
+  uint32_t gcur[kMaxNb1];
+  int64_t ws[33];
+};
+
+__global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_constant__ GroupArgs g) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  ScatterSmem &S = *reinterpret_cast<ScatterSmem *>(smraw);
+  const int nb = (int)g.plan.nb1;
   const int bits = g.plan.bits1;
   for (int64_t k = blockIdx.x; k < g.plan.nchunks; k += gridDim.x) {
     const int j = g.plan.chunk_trial[k];
-    const uint32_t *pre = g.counts + k * nb;
-    const uint32_t *bst = g.bstart1 + (int64_t)j * nb;
-    __syncthreads();
-    for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) cur[i] = bst[i] + pre[i];
-    __syncthreads();
     const int64_t i0 = g.plan.chunk_i0[k];
     const int64_t in0 = g.plan.in_base[j] + i0;
     const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];   // scratch segment start
     const int len = g.plan.chunk_len[k];
-    for (int base = threadIdx.x; base < len; base += blockDim.x * kItems) {
-      uint64_t kk[kItems];
-      uint32_t vv[kItems];
+    const uint32_t *pre = g.counts + k * nb;
+    const uint32_t *bst = g.bstart1 + (int64_t)j * nb;
+    for (int b = threadIdx.x; b < nb; b += blockDim.x) S.gcur[b] = bst[b] + pre[b];
+    {
+      uint64_t kk[kPerLane];
 #pragma unroll
-      for (int u = 0; u < kItems; ++u) {
-        const int i = base + u * blockDim.x;
-        if (i < len) {
-          kk[u] = g.keys[in0 + i];
-          vv[u] = val_at(g, in0 + i, i0 + i);
-        }
+      for (int u = 0; u < kPerLane; ++u) {
+        const int e = threadIdx.x + u * kSThreads;
+        if (e < len) kk[u] = g.keys[in0 + e];
       }
 #pragma unroll
-      for (int u = 0; u < kItems; ++u) {
-        const int i = base + u * blockDim.x;
-        if (i < len) {
-          const uint32_t pos = atomicAdd(&cur[top_bits(kk[u], bits)], 1u);
-          g.akeys[sseg + pos] = kk[u];
-          g.avals[sseg + pos] = vv[u];
-        }
+      for (int u = 0; u < kPerLane; ++u) {
+        const int e = threadIdx.x + u * kSThreads;
+        if (e < len) S.K[e] = kk[u];
       }
     }
+    __syncthreads();
+    stable_split(S.K, len, nb, [&](uint64_t key) { return top_bits(key, bits); }, S.cnt, S.sbst,
+                 S.ws, [&](int e, int p, uint32_t b) {
+                   const int64_t o = sseg + S.gcur[b] + (p - (int)S.sbst[b]);
+                   g.akeys[o] = S.K[e];
+                   g.avals[o] = val_at(g, in0 + e, i0 + e);
+                 });
   }
 }
 
-// ---- 4. second-level scatter (one CTA per coarse bucket) ----------------------
-__global__ void __launch_bounds__(kGThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
-  __shared__ uint32_t cnt[1 << (kMaxBits - kCoarseBits)];
-  __shared__ int64_t ws[33];
+// ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
+struct Scatter2Smem {
+  uint64_t K[kChunk];
+  uint16_t cnt[kWarps * kMaxNb2];
+  uint32_t sbst[kMaxNb2];
+  uint32_t tot[kMaxNb2];
+  uint32_t gcur[kMaxNb2];
+  int64_t ws[33];
+};
+
+__global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  Scatter2Smem &S = *reinterpret_cast<Scatter2Smem *>(smraw);
   const int64_t q1 = blockIdx.x;                 // (trial, coarse bucket)
   const int64_t nb1 = g.plan.nb1;
   const int j = (int)(q1 / nb1);
@@ -160,53 +260,52 @@ __global__ void __launch_bounds__(kGThreads, 2) scatter2_kernel(const __grid_con
   const int64_t n = g.bsize1[q1];
   const uint64_t *__restrict__ K = g.akeys + sseg + st1;
   const uint32_t *__restrict__ V = g.avals + sseg + st1;
-  for (int i = threadIdx.x; i < nb2; i += blockDim.x) cnt[i] = 0;
+  auto fine = [&](uint64_t key) { return top_bits(key, bits) & mask2; };
+  // fine-bucket totals (order-free), starts, sizes
+  for (int i = threadIdx.x; i < nb2; i += blockDim.x) S.tot[i] = 0;
   __syncthreads();
-  for (int64_t base = threadIdx.x; base < n; base += (int64_t)blockDim.x * kItems) {
-    uint64_t kk[kItems];
-#pragma unroll
-    for (int u = 0; u < kItems; ++u) {
-      const int64_t i = base + u * blockDim.x;
-      kk[u] = i < n ? K[i] : 0;
-    }
-#pragma unroll
-    for (int u = 0; u < kItems; ++u)
-      if (base + u * (int64_t)blockDim.x < n) atomicAdd(&cnt[top_bits(kk[u], bits) & mask2], 1u);
-  }
+  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&S.tot[fine(K[i])], 1u);
   __syncthreads();
-  // final bucket starts / sizes of this coarse bucket's sub-buckets
   {
     const int d = threadIdx.x;
-    const int64_t v = d < nb2 ? cnt[d] : 0;
-    int64_t tot;
-    const int64_t ex = block_excl_scan<int64_t>(v, ws, &tot);
+    const int64_t v = d < nb2 ? S.tot[d] : 0;
+    int64_t all;
+    const int64_t ex = block_excl_scan<int64_t>(v, S.ws, &all);
     if (d < nb2) {
       const int64_t qf = (int64_t)j * g.plan.nbins + ((int64_t)b1 << bits2) + d;
       g.bstart[qf] = st1 + (uint32_t)ex;
       g.bsize[qf] = (uint32_t)v;
-      cnt[d] = st1 + (uint32_t)ex;
+      S.gcur[d] = st1 + (uint32_t)ex;
     }
   }
   __syncthreads();
-  for (int64_t base = threadIdx.x; base < n; base += (int64_t)blockDim.x * kItems) {
-    uint64_t kk[kItems];
-    uint32_t vv[kItems];
+  for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
+    const int len = (int)min((int64_t)kChunk, n - c0);
+    {
+      uint64_t kk[kPerLane];
 #pragma unroll
-    for (int u = 0; u < kItems; ++u) {
-      const int64_t i = base + u * blockDim.x;
-      if (i < n) {
-        kk[u] = K[i];
-        vv[u] = V[i];
+      for (int u = 0; u < kPerLane; ++u) {
+        const int e = threadIdx.x + u * kSThreads;
+        if (e < len) kk[u] = K[c0 + e];
+      }
+#pragma unroll
+      for (int u = 0; u < kPerLane; ++u) {
+        const int e = threadIdx.x + u * kSThreads;
+        if (e < len) S.K[e] = kk[u];
       }
     }
-#pragma unroll
-    for (int u = 0; u < kItems; ++u) {
-      if (base + u * (int64_t)blockDim.x < n) {
-        const uint32_t pos = atomicAdd(&cnt[top_bits(kk[u], bits) & mask2], 1u);
-        g.bkeys[sseg + pos] = kk[u];
-        g.bvals[sseg + pos] = vv[u];
-      }
+    __syncthreads();
+    stable_split(S.K, len, nb2, fine, S.cnt, S.sbst, S.ws, [&](int e, int p, uint32_t d) {
+      const int64_t o = sseg + S.gcur[d] + (p - (int)S.sbst[d]);
+      g.bkeys[o] = S.K[e];
+      g.bvals[o] = V[c0 + e];
+    });
+    // advance the fine cursors by this sub-chunk's counts
+    for (int d = threadIdx.x; d < nb2; d += blockDim.x) {
+      const uint32_t end = d + 1 < nb2 ? S.sbst[d + 1] : (uint32_t)len;
+      S.gcur[d] += end - S.sbst[d];
     }
+    __syncthreads();
   }
 }
 
@@ -230,13 +329,15 @@ __global__ void sum_i32_kernel(const int32_t *__restrict__ a, int64_t n, unsigne
 
 }  // namespace
 
+int64_t group_chunk_pairs() { return kChunk; }
+
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1) {
-  // final buckets of <= ~4K pairs on average (the shared-memory sort holds 8K)
+  // final buckets of <= ~2K pairs on average (the shared-memory sort holds 4K)
   // test hook SG_GROUP_TARGET: smaller target buckets (forces the two-level
   // partition and the big-bucket path on graphs the oracle can check)
   const char *e = getenv("SG_GROUP_TARGET");
-  int64_t target = e ? atoll(e) : 4096;
-  if (target <= 0) target = 4096;
+  int64_t target = e ? atoll(e) : 2048;
+  if (target <= 0) target = 2048;
   int b = 0;
   while ((maxseg >> b) > target && b < kMaxBits) ++b;
   *bits = b;
@@ -262,8 +363,11 @@ cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
 
 cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
-  const size_t smem = (size_t)g.plan.nb1 * sizeof(uint32_t);
-  const int grid = (int)std::min<int64_t>(num_sms, g.plan.nchunks);
+  const size_t smem = sizeof(ScatterSmem);
+  cudaError_t e = cudaFuncSetAttribute(scatter_kernel,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * 2, g.plan.nchunks);
   scatter_kernel<<<grid, kSThreads, smem, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
@@ -272,7 +376,11 @@ cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
 cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   const int64_t nq1 = (int64_t)g.plan.c * g.plan.nb1;
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
-  scatter2_kernel<<<(unsigned)nq1, kGThreads, 0, st>>>(g);
+  const size_t smem = sizeof(Scatter2Smem);
+  cudaError_t e = cudaFuncSetAttribute(scatter2_kernel,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  scatter2_kernel<<<(unsigned)nq1, kSThreads, smem, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }

@@ -1,18 +1,22 @@
 // kernels_local.cu — sort inside one key bucket and run-length segmentation:
 // the second half of the per-trial grouping (AMB-5).
 //
-// local_kernel: persistent, one CTA (1024 threads) per SM, buckets of up to
-// 8192 pairs double-buffered into shared memory with cp.async.  Per bucket:
-//   * counting sort on the next <= 11 key bits (sub-bins of ~1-2 pairs);
-//   * element-parallel placement: every pair counts the pairs of its sub-bin
-//     that precede it in (key, member) order -> its position; it opens a group
-//     (head bit) iff no pair with an equal key has a smaller member;
-//   * sub-bins with > 64 pairs (long runs of one key = big groups) are
-//     bitonic-sorted by a warp (<= 256) or by the whole CTA;
-//   * members are written at bucket offset + position, the head bits as
-//     32-bit words (atomicOr on the two words shared with neighbours).
-// big_kernel: buckets above 8192 pairs, one CTA each, bitonic sort in global
-// (L2-resident) memory.
+// The partition (kernels_group.cu) is stable, so inside a bucket the pairs
+// of one trial are still in generator order and a STABLE sort by key alone
+// yields the canonical (key, member) order.
+//
+// local_kernel: persistent CTAs of 8 warps (3 per SM overlap each other's
+// loads), one bucket of up to 4096 pairs at a time in shared memory:
+//   * two stable LSD multi-split passes on the 16 key bits after the bucket
+//     bits (8 bits each; warp segments, __match_any_sync ranks, a bin-major
+//     [digit][warp] counter matrix turned into starts by one block scan): the
+//     pairs of one group stay together and in member order;
+//   * the rare runs where distinct keys share those 16 bits out of order get
+//     a stable insertion sort by key;
+//   * members are written in sorted order (coalesced), one head bit per group
+//     start (ballot per 32 positions).
+// big_kernel: buckets above 4096 pairs, one CTA each, bitonic sort by the
+// total order (key, member) in global (L2-resident) memory.
 #include <algorithm>
 
 #include "group_common.cuh"
@@ -24,48 +28,94 @@ namespace sg {
 
 namespace {
 
-using grp::bitonic_idx;
 using grp::bucket_extent;
 using grp::pair_less;
 
-constexpr int kLocalCap = 8192;
-constexpr int kLThreads = 1024;
-constexpr int kMaxSubBits = 11;
-constexpr int kNSubMax = 1 << kMaxSubBits;
-constexpr int kRankMax = 64;         // sub-bins up to this size: element-parallel ranks
-constexpr int kWarpSortMax = 256;    // then warp bitonic, then CTA bitonic
-constexpr int kMaxList = 64;
+constexpr int kLocalCap = 4096;
+constexpr int kLThreads = 256;
+constexpr int kLWarps = kLThreads / 32;
+constexpr int kPerLane = kLocalCap / kLThreads;   // 16
+constexpr int kDigitBits = 8;                     // two stable LSD passes = 16 key bits
+constexpr int kDigits = 1 << kDigitBits;
+constexpr int kCntPerThread = kDigits * kLWarps / kLThreads;   // 8
 
 struct LocalSmem {
-  uint64_t K[2][kLocalCap];
-  uint32_t V[2][kLocalCap];
-  uint16_t perm[kLocalCap];
-  uint32_t sub[kNSubMax];
+  uint64_t K[kLocalCap];
+  uint32_t V[kLocalCap];
+  uint16_t perm[2][kLocalCap];
+  uint16_t cnt[kDigits * kLWarps];   // bin-major: [digit][warp]
+  uint32_t peers[kLocalCap];         // match masks (warp segments)
+  uint32_t nfix;
+  uint32_t fix[64];
   uint32_t hb[kLocalCap / 32 + 2];
   int64_t ws[33];
-  uint32_t run_st[kMaxList];
-  uint32_t run_n[kMaxList];
-  int nrun;
 };
+static_assert(kCntPerThread == 8, "counter scan assumes 8 per thread");
 
-__device__ __forceinline__ void cp_async8(void *sdst, const void *gsrc) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(sdst);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gsrc));
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
 }
-__device__ __forceinline__ void cp_async4(void *sdst, const void *gsrc) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(sdst);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gsrc));
-}
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-__device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;\n" ::); }
 
-__device__ __forceinline__ void prefetch_bucket(LocalSmem &S, int buf, const GroupArgs &g,
-                                                int64_t sbase, int64_t n) {
-  if (n > kLocalCap) n = 0;
-  for (int i = threadIdx.x; i < n; i += blockDim.x) {
-    cp_async8(&S.K[buf][i], g.bkeys + sbase + i);
-    cp_async4(&S.V[buf][i], g.bvals + sbase + i);
+// One stable multi-split pass over n <= 4096 elements: warp w owns the
+// positions [w*seg, (w+1)*seg) of the current order src (identity if null)
+// and writes the new order to dst, stable on digit(key).
+template <typename DIG>
+__device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *src, uint16_t *dst,
+                                         DIG digit) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint32_t lt = lanemask_lt();
+  const int seg = (n + kLWarps - 1) / kLWarps;     // <= 512
+  reinterpret_cast<uint4 *>(S.cnt)[threadIdx.x] = make_uint4(0, 0, 0, 0);
+  __syncthreads();
+  uint32_t *pr = S.peers + w * kPerLane * 32;     // match masks of this warp
+  const int seg_lo = w * seg, seg_hi = min(n, seg_lo + seg);
+  for (int pos = seg_lo + lane; pos - lane < seg_hi; pos += 32) {   // warp-uniform trip count
+    const bool valid = pos < seg_hi;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    if (valid) {
+      const uint32_t dg = digit(S.K[src ? src[pos] : pos]);
+      const uint32_t m = __match_any_sync(vm, dg);
+      pr[pos - seg_lo] = m;
+      if ((m & lt) == 0) S.cnt[dg * kLWarps + w] += (uint16_t)__popc(m);
+    }
   }
+  __syncthreads();
+  {
+    // exclusive scan of the bin-major counters (8 per thread)
+    uint4 *c4 = reinterpret_cast<uint4 *>(S.cnt);
+    uint4 v = c4[threadIdx.x];
+    uint16_t *c = reinterpret_cast<uint16_t *>(&v);
+    uint32_t s = 0, run[kCntPerThread];
+#pragma unroll
+    for (int x = 0; x < kCntPerThread; ++x) {
+      run[x] = s;
+      s += c[x];
+    }
+    int64_t tot;
+    const int64_t ex = block_excl_scan<int64_t>((int64_t)s, S.ws, &tot);
+#pragma unroll
+    for (int x = 0; x < kCntPerThread; ++x) c[x] = (uint16_t)(ex + run[x]);
+    c4[threadIdx.x] = v;
+  }
+  __syncthreads();
+  for (int pos = seg_lo + lane; pos - lane < seg_hi; pos += 32) {
+    const bool valid = pos < seg_hi;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    if (valid) {
+      const uint16_t el = src ? src[pos] : (uint16_t)pos;
+      const uint32_t dg = digit(S.K[el]);
+      const uint32_t m = pr[pos - seg_lo];
+      const uint32_t rank = __popc(m & lt);
+      const uint32_t base = S.cnt[dg * kLWarps + w];
+      __syncwarp(vm);
+      if (rank == 0) S.cnt[dg * kLWarps + w] = (uint16_t)(base + __popc(m));
+      __syncwarp(vm);
+      dst[base + rank] = el;
+    }
+  }
+  __syncthreads();
 }
 
 // Head-bit words of output positions [gbase, gbase + n) from the bucket-local
@@ -91,141 +141,101 @@ __device__ __forceinline__ void store_heads(uint32_t *head, const uint32_t *hb, 
   }
 }
 
-__global__ void __launch_bounds__(kLThreads, 1) local_kernel(const __grid_constant__ GroupArgs g) {
+__global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   LocalSmem &S = *reinterpret_cast<LocalSmem *>(smraw);
   const int64_t nq = (int64_t)g.plan.c * g.plan.nbins;
   const int bits = g.plan.bits;
   const int64_t obase = g.plan.seg[0];     // scratch -> output position
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
-  int64_t q = blockIdx.x;
-  int cur = 0;
-  int64_t sb = 0, n64 = 0;
-  if (q < nq) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int64_t q = blockIdx.x; q < nq; q += gridDim.x) {
+    int64_t sb, n64;
     bucket_extent(g, q, sb, n64);
-    prefetch_bucket(S, 0, g, sb, n64);
-  }
-  cp_commit();
-  for (; q < nq; q += gridDim.x) {
-    const int64_t qn = q + gridDim.x;
-    int64_t sbn = 0, nn = 0;
-    if (qn < nq) {
-      bucket_extent(g, qn, sbn, nn);
-      prefetch_bucket(S, cur ^ 1, g, sbn, nn);
-    }
-    cp_commit();
-    cp_wait1();
-    __syncthreads();
+    if (n64 == 0) continue;
     if (n64 > kLocalCap) {
       if (threadIdx.x == 0) g.big_list[atomicAdd(g.big_count, 1u)] = (uint32_t)q;
-    } else if (n64 > 0) {
-      const int n = (int)n64;
-      const uint64_t *K = S.K[cur];
-      const uint32_t *V = S.V[cur];
-      int sbits = 1;
-      while ((1 << sbits) < n && sbits < kMaxSubBits) ++sbits;
-      const int nsub = 1 << sbits;
-      const int nhw = (n + 31) >> 5;
-      for (int i = threadIdx.x; i < nsub; i += blockDim.x) S.sub[i] = 0;
-      for (int i = threadIdx.x; i < nhw; i += blockDim.x) S.hb[i] = 0;
-      if (threadIdx.x == 0) S.nrun = 0;
-      __syncthreads();
-      auto subof = [&](uint64_t key) { return (uint32_t)((key << bits) >> (64 - sbits)); };
-      for (int i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&S.sub[subof(K[i])], 1u);
-      __syncthreads();
-      {
-        const int per = (nsub + blockDim.x - 1) / blockDim.x;   // <= 2
-        const int b0 = threadIdx.x * per;
-        uint32_t v0 = (per > 0 && b0 < nsub) ? S.sub[b0] : 0u;
-        uint32_t v1 = (per > 1 && b0 + 1 < nsub) ? S.sub[b0 + 1] : 0u;
-        int64_t tot;
-        const int64_t ex = block_excl_scan<int64_t>((int64_t)v0 + v1, S.ws, &tot);
-        if (per > 0 && b0 < nsub) S.sub[b0] = (uint32_t)ex;
-        if (per > 1 && b0 + 1 < nsub) S.sub[b0 + 1] = (uint32_t)(ex + v0);
-      }
-      __syncthreads();
-      for (int i = threadIdx.x; i < n; i += blockDim.x)
-        S.perm[atomicAdd(&S.sub[subof(K[i])], 1u)] = (uint16_t)i;
-      __syncthreads();
-      // S.sub[d] is now the end of sub-bin d; element-parallel placement
-      const int64_t gbase = obase + sb;
-      for (int i = threadIdx.x; i < n; i += blockDim.x) {
-        const uint64_t ki = K[i];
-        const uint32_t vi = V[i];
-        const uint32_t d = subof(ki);
-        const int en = (int)S.sub[d];
-        const int st = d ? (int)S.sub[d - 1] : 0;
-        const int m = en - st;
-        int pos, eq = 0;
-        if (m == 1) {
-          pos = st;
-        } else if (m <= kRankMax) {
-          int rank = 0;
-          for (int x = st; x < en; ++x) {
-            const int e = S.perm[x];
-            const uint64_t ke = K[e];
-            const uint32_t ve = V[e];
-            rank += pair_less(ke, ve, ki, vi);
-            eq += (ke == ki) & (ve < vi);
-          }
-          pos = st + rank;
-        } else {
-          if (S.perm[st] == i) {                   // one representative registers the run
-            const int s = atomicAdd(&S.nrun, 1);
-            if (s < kMaxList) {
-              S.run_st[s] = st;
-              S.run_n[s] = m;
-            }
-          }
-          continue;
+      continue;
+    }
+    const int n = (int)n64;
+    for (int i = threadIdx.x; i < n; i += kLThreads) {
+      const unsigned sk = (unsigned)__cvta_generic_to_shared(&S.K[i]);
+      const unsigned sv = (unsigned)__cvta_generic_to_shared(&S.V[i]);
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sk), "l"(g.bkeys + sb + i));
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sv), "l"(g.bvals + sb + i));
+    }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_all;\n" ::);
+    // (lsd_pass begins with a barrier after zeroing its counters)
+    lsd_pass(S, n, nullptr, S.perm[0],
+             [&](uint64_t key) { return (uint32_t)((key << (bits + 8)) >> 56); });
+    lsd_pass(S, n, S.perm[0], S.perm[1],
+             [&](uint64_t key) { return (uint32_t)((key << bits) >> 56); });
+    const uint16_t *pm = S.perm[1];
+    const uint64_t *K = S.K;
+    auto d16 = [&](uint64_t key) { return (uint32_t)((key << bits) >> 48); };
+    // ---- rare: distinct keys sharing the 16 bits out of key order -> a
+    // stable insertion sort of that run (registered once via its start bit)
+    for (int i = threadIdx.x; i < (kLocalCap / 32 + 2); i += blockDim.x) S.hb[i] = 0;
+    if (threadIdx.x == 0) S.nfix = 0;
+    __syncthreads();
+    for (int p = threadIdx.x + 1; p < n; p += blockDim.x) {
+      const uint64_t kp = K[pm[p]];
+      if (kp < K[pm[p - 1]]) {
+        const uint32_t dp = d16(kp);
+        int a = p - 1;
+        while (a > 0 && d16(K[pm[a - 1]]) == dp) --a;
+        const uint32_t bit = 1u << (a & 31);
+        if (!(atomicOr(&S.hb[a >> 5], bit) & bit)) {
+          const uint32_t s = atomicAdd(&S.nfix, 1u);
+          if (s < 64) S.fix[s] = (uint32_t)a;
         }
-        g.members[gbase + pos] = vi;
-        if (eq == 0) atomicOr(&S.hb[pos >> 5], 1u << (pos & 31));
       }
-      __syncthreads();
-      const int nrun = S.nrun;
-      if (nrun > 0) {
-        if (nrun > kMaxList) {
-          // more long runs than list slots: sort the whole bucket and place it
-          bitonic_idx(S.perm, n, K, V, threadIdx.x, blockDim.x, [] { __syncthreads(); });
-          for (int i = threadIdx.x; i < nhw; i += blockDim.x) S.hb[i] = 0;
-          __syncthreads();
-          for (int p = threadIdx.x; p < n; p += blockDim.x) {
-            const int e = S.perm[p];
-            g.members[gbase + p] = V[e];
-            if (p == 0 || K[S.perm[p - 1]] != K[e]) atomicOr(&S.hb[p >> 5], 1u << (p & 31));
-          }
-        } else {
-          for (int x = wid; x < nrun; x += nwarp) {
-            if (S.run_n[x] <= kWarpSortMax)
-              bitonic_idx(S.perm + S.run_st[x], (int)S.run_n[x], K, V, lane, 32, [] { __syncwarp(); });
-          }
-          for (int x = 0; x < nrun; ++x) {
-            if (S.run_n[x] > kWarpSortMax)
-              bitonic_idx(S.perm + S.run_st[x], (int)S.run_n[x], K, V, threadIdx.x, blockDim.x,
-                          [] { __syncthreads(); });
-          }
-          __syncthreads();
-          for (int x = 0; x < nrun; ++x) {
-            const int st = (int)S.run_st[x], m = (int)S.run_n[x];
-            for (int t = threadIdx.x; t < m; t += blockDim.x) {
-              const int p = st + t;
-              const int e = S.perm[p];
-              g.members[gbase + p] = V[e];
-              if (t == 0 || K[S.perm[p - 1]] != K[e]) atomicOr(&S.hb[p >> 5], 1u << (p & 31));
-            }
-          }
-        }
-        __syncthreads();
-      }
-      store_heads(g.head, S.hb, gbase, n);
     }
     __syncthreads();
-    cur ^= 1;
-    sb = sbn;
-    n64 = nn;
+    const uint32_t nfix = S.nfix;
+    if (nfix > 64) {
+      // pathological: one stable insertion sort of everything
+      if (threadIdx.x == 0) {
+        uint16_t *q2 = S.perm[1];
+        for (int x = 1; x < n; ++x) {
+          const uint16_t e = q2[x];
+          const uint64_t ke = K[e];
+          int y = x - 1;
+          while (y >= 0 && ke < K[q2[y]]) { q2[y + 1] = q2[y]; --y; }
+          q2[y + 1] = e;
+        }
+      }
+    } else if (threadIdx.x < (int)nfix) {
+      uint16_t *q2 = S.perm[1];
+      const int a = (int)S.fix[threadIdx.x];
+      const uint32_t da = d16(K[q2[a]]);
+      int b = a + 1;
+      while (b < n && d16(K[q2[b]]) == da) ++b;
+      for (int x = a + 1; x < b; ++x) {
+        const uint16_t e = q2[x];
+        const uint64_t ke = K[e];
+        int y = x - 1;
+        while (y >= a && ke < K[q2[y]]) { q2[y + 1] = q2[y]; --y; }   // strict: stable
+        q2[y + 1] = e;
+      }
+    }
+    __syncthreads();
+    // ---- members in sorted order + head bits (ballot per 32 positions)
+    const int64_t gbase = obase + sb;
+    for (int p0 = w * 32; p0 < n; p0 += blockDim.x) {
+      const int p = p0 + lane;
+      bool head = false;
+      if (p < n) {
+        const int e = pm[p];
+        g.members[gbase + p] = S.V[e];
+        head = (p == 0) || K[pm[p - 1]] != K[e];
+      }
+      const uint32_t hw = __ballot_sync(0xffffffffu, head);
+      if (lane == 0) S.hb[p0 >> 5] = hw;
+    }
+    __syncthreads();
+    store_heads(g.head, S.hb, gbase, n);
+    __syncthreads();
   }
-  asm volatile("cp.async.wait_all;\n" ::);
 }
 
 // ---- big buckets: one CTA, bitonic in global memory ---------------------------
@@ -280,7 +290,11 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   cudaError_t e = cudaFuncSetAttribute(local_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)smem);
   if (e != cudaSuccess) return e;
-  const int grid = (int)std::min<int64_t>((int64_t)num_sms, nq);
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_kernel, kLThreads, smem);
+  if (e != cudaSuccess) return e;
+  per_sm = std::max(per_sm, 1);
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, nq);
   local_kernel<<<grid, kLThreads, smem, st>>>(g);
   ++g_launches;
   return cudaGetLastError();

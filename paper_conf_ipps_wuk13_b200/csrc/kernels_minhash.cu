@@ -102,6 +102,23 @@ __device__ __forceinline__ void scan_all(const uint32_t *nb, int len, uint32_t a
   }
 }
 
+// Short rows (the staged tile pads each row to a multiple of 4): branch-free,
+// padding slots masked to +infinity, no remainder loop.
+template <int S>
+__device__ __forceinline__ void scan_short(const uint32_t *nb, int len, uint32_t a, uint32_t b,
+                                           uint32_t (&m)[S]) {
+  const uint4 *nb4 = reinterpret_cast<const uint4 *>(nb);
+  const int nq = (len + 3) >> 2;
+  for (int q = 0; q < nq; ++q) {
+    const uint4 v = nb4[q];
+    const int e = q << 2;
+    insert_min<S>(m, m31_hash(a, b, v.x));
+    insert_min<S>(m, e + 1 < len ? m31_hash(a, b, v.y) : 0xFFFFFFFFu);
+    insert_min<S>(m, e + 2 < len ? m31_hash(a, b, v.z) : 0xFFFFFFFFu);
+    insert_min<S>(m, e + 3 < len ? m31_hash(a, b, v.w) : 0xFFFFFFFFu);
+  }
+}
+
 template <int S>
 __device__ __forceinline__ void scan_any(const uint32_t *nb, int len, int part, int p, uint32_t a,
                                          uint32_t b, uint32_t (&m)[S]) {
@@ -227,7 +244,8 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
           uint32_t m[S];
 #pragma unroll
           for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
-          scan_any<S>(nb + sOff[w][rr], rl, part, p, A, B, m);
+          if (p == 1 && rl <= 24) scan_short<S>(nb + sOff[w][rr], rl, A, B, m);
+          else scan_any<S>(nb + sOff[w][rr], rl, part, p, A, B, m);
           // merge the p partial lists of a trial (lanes tl, tl + T, ...)
           for (int o = T; o < 32; o <<= 1) {
             uint32_t x[S];

@@ -159,4 +159,6 @@ struct sg_graph {
   std::vector<std::pair<int, int>> st[sg::kNumStages];
   int64_t mem_budget = 0;       // test hook: cap on planned bytes (0 = free HBM)
   int64_t bytes_live = 0;       // device bytes currently held by this handle
+  std::vector<sg::DBuf> cache;  // freed blocks kept for reuse (best fit)
+  int64_t bytes_cached = 0;
 };
