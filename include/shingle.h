@@ -118,11 +118,11 @@ SG_API sg_status group_by_shingle(sg_graph *g);
 /* (mode 0, AMB-9) or that generated its first-level shingles (mode 1).     */
 /*   labels     host int32[n], caller-allocated; labels[v] = smallest vertex */
 /*              of v's cluster (AMB-10); clusters smaller than min_size are  */
-/*              reported as singletons (labels[v] = v).  Filled on rank 0;   */
-/*              other ranks may pass NULL.                                   */
+/*              reported as singletons (labels[v] = v).                      */
 /*   n_clusters receives the number of clusters with >= max(2, min_size)     */
 /*              vertices (may be NULL).                                      */
-/* Host work, outside the timed hot path.  Requires state GROUPED2.          */
+/* Host work, outside the timed hot path.  Requires state GROUPED2 and      */
+/* world == 1 (SG_ESTATE otherwise: gather G_II with sg_get_groups).         */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
                                  int64_t *n_clusters);
@@ -148,6 +148,8 @@ SG_API const char *sg_last_error(const sg_graph *g);
 /* DESIGN.md §6.3), 0, 0.  Global counts are summed over ranks.  The        */
 /* environment variable SG_MEM_BUDGET (bytes, read at create) caps the HBM   */
 /* the planner assumes, to exercise the chunked paths on small graphs.      */
+/* world > 1: collective (every rank calls it; it sums the counts once per   */
+/* level), like shingle_pass and group_by_shingle.  Other getters are local. */
 SG_API sg_status sg_get_counts(const sg_graph *g, int64_t counts[16]);
 
 /* Shingle matrix of pass `level` (1 or 2) on this rank: ids[rows x c]      */
@@ -181,6 +183,19 @@ SG_API sg_status sg_get_stage_ms(const sg_graph *g, float *ms, int32_t cap, int3
 typedef struct sg_loopback sg_loopback;
 SG_API sg_status sg_loopback_create(int32_t world, sg_loopback **out);
 SG_API void sg_loopback_destroy(sg_loopback *lb);
+
+/* NCCL backend: rank 0 creates the 128-byte ncclUniqueId that every rank    */
+/* passes in sg_dist.nccl_uid (broadcast it, e.g. with torch.distributed).   */
+/* SG_ENCCL if libnccl.so.2 cannot be loaded.                                */
+SG_API sg_status sg_nccl_unique_id(uint8_t *out128);
+
+/* Canonical pass-II dense index: given the all-gathered      */
+/* counts all[r * c1 + j] of S1' rows of pass-I trial j on rank r, the local */
+/* rows of trial j on `rank` are [first[j], first[j+1]) and row i of trial j */
+/* gets k = i + off[j].  first[c1 + 1], off[c1]; returns |S1'| in *total.     */
+/* Pure host code (testable without GPU).                                    */
+SG_API sg_status sg_s1p_offsets(int32_t world, int32_t rank, int32_t c1, const int64_t *all,
+                                int64_t *first, int64_t *off, int64_t *total);
 
 /* Host-side vertex-range partition used by create: splits   */
 /* [0, n) into `world` contiguous ranges balancing sum(deg + kappa).  bounds */

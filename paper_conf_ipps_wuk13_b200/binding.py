@@ -66,6 +66,8 @@ def lib() -> C.CDLL:
         "sg_loopback_create": (st, [i32, C.POINTER(vp)]),
         "sg_loopback_destroy": (None, [vp]),
         "sg_partition_rows": (st, [i64, vp, i32, i64, vp]),
+        "sg_nccl_unique_id": (st, [vp]),
+        "sg_s1p_offsets": (st, [i32, i32, i32, vp, vp, vp, vp]),
         "sg_version": (C.c_char_p, []),
     }
     for name, (rt, args) in sig.items():
@@ -213,6 +215,28 @@ def sg_loopback_create(world: int):
 
 def sg_loopback_destroy(lb):
     lib().sg_loopback_destroy(lb)
+
+
+def sg_nccl_unique_id() -> bytes:
+    """128-byte ncclUniqueId (rank 0 creates it; broadcast it to the others)."""
+    buf = C.create_string_buffer(128)
+    _check(lib().sg_nccl_unique_id(buf))
+    return buf.raw
+
+
+nccl_unique_id = sg_nccl_unique_id
+
+
+def sg_s1p_offsets(all_counts, rank: int):
+    """all_counts int64[world, c1] -> (first[c1+1], off[c1], total): canonical S1' index map."""
+    a = np.ascontiguousarray(all_counts, np.int64)
+    world, c1 = a.shape
+    first = np.zeros(c1 + 1, np.int64)
+    off = np.zeros(max(c1, 1), np.int64)
+    tot = C.c_int64()
+    _check(lib().sg_s1p_offsets(world, rank, c1, a.ctypes.data, first.ctypes.data, off.ctypes.data,
+                                C.byref(tot)))
+    return first, off[:c1], tot.value
 
 
 def sg_version() -> str:

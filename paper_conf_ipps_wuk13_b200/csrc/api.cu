@@ -155,25 +155,32 @@ void st_clear(sg_graph *g) {
   g->ev_next = 0;
 }
 
+// `collective` calls (pass, group) run exchange steps on world > 1: a rank
+// that fails inside one breaks a loopback group so its peers return too.
 template <typename F>
-sg_status guarded(sg_graph *g, F &&f) {
+sg_status guarded(sg_graph *g, F &&f, bool collective = false) {
   if (!g) {
     t_err = "null handle";
     return SG_EINVAL;
   }
-  if (g->state == kPoisoned) return g->poison;
-  try {
-    int dev = -1;
-    cudaGetDevice(&dev);
-    if (dev != g->device) CK(cudaSetDevice(g->device));
-    f();
-    return SG_OK;
-  } catch (const Fail &x) {
-    return x.st;
-  } catch (const std::bad_alloc &) {
-    set_err(g, "host allocation failed");
-    return SG_ENOMEM;
+  sg_status st = SG_OK;
+  if (g->state == kPoisoned) {
+    st = g->poison;
+  } else {
+    try {
+      int dev = -1;
+      cudaGetDevice(&dev);
+      if (dev != g->device) CK(cudaSetDevice(g->device));
+      f();
+    } catch (const Fail &x) {
+      st = x.st;
+    } catch (const std::bad_alloc &) {
+      set_err(g, "host allocation failed");
+      st = SG_ENOMEM;
+    }
   }
+  if (st != SG_OK && collective && g->xch) exchange_abort(g->xch);
+  return st;
 }
 
 void free_pass(sg_graph *g, PassOut &p) {
@@ -185,6 +192,7 @@ void free_pass(sg_graph *g, PassOut &p) {
 void free_groups(sg_graph *g, Groups &q) {
   dfree(g, q.members);
   dfree(g, q.head);
+  dfree(g, q.okeys);
   q = Groups();
 }
 
@@ -248,7 +256,15 @@ void plan_pass(sg_graph *g, PassOut &P) {
   const double avail = (double)avail_bytes(g);
   int64_t ct = (int64_t)((avail - members - keys_t * c) / scr_t);
   P.deferred = false;
-  if (ct < 1) {
+  if (g->world > 1) {
+    // multi-rank: all keys are kept until their exchange (eager), sorted keys
+    // are kept for the getters, send + receive buffers per chunk; every rank
+    // uses the same trial chunks (the exchange rounds must match)
+    const double mr_t = scr_t + 24.0 * (double)nr + 8.0 * (double)nr;
+    ct = (int64_t)((avail - members - keys_t * c) / mr_t);
+    ct = exchange_min(g, std::max<int64_t>(ct, 0));
+    if (ct < 1) fail(g, SG_ENOMEM, "multi-rank pass needs all keys resident; not enough HBM");
+  } else if (ct < 1) {
     ct = (int64_t)((avail - members) / (keys_t + scr_t));
     P.deferred = true;
     if (ct < 1) {
@@ -316,12 +332,58 @@ double scratch_per_pair(int64_t maxseg) {
   return b == b1 ? 12.5 : 24.5;
 }
 
-// Group the pairs of trials [t0, t0 + nt) whose keys are `keys` ([nt][stride])
-// into out.members / out.head at the global positions seg_all[t].
-void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, int32_t nt,
-                 const std::vector<int64_t> &seg_all, const uint32_t *vals, const uint32_t *rowid,
-                 uint32_t val_base, Groups &out, GroupScratch &S, DBuf *free_after_scatter,
-                 int st_hist, int st_scatter, int st_local) {
+// A contiguous run of pre-group pairs of one (local) trial: keys / explicit
+// values at [in0, in0 + len), generator rows row0.. (implicit values).
+struct Piece {
+  int32_t trial;
+  int64_t in0, len, row0;
+};
+
+void upload(sg_graph *g, DBuf &b, const void *h, size_t bytes) {
+  if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
+  if (bytes) CK(cudaMemcpyAsync(b.p, h, bytes, cudaMemcpyHostToDevice, g->stream));
+}
+
+void need(sg_graph *g, DBuf &b, size_t bytes) {
+  if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
+}
+
+// Chunk table of a partition over `nt` trials: pieces (ordered by trial, then
+// input order) cut into chunks of <= group_chunk_pairs() pairs.
+int64_t build_chunks(sg_graph *g, const std::vector<Piece> &pieces, int32_t nt, GroupScratch &S) {
+  const int64_t CH = group_chunk_pairs();
+  std::vector<int64_t> ci0, cin;
+  std::vector<int32_t> clen, ctr, tc0((size_t)nt + 1, 0);
+  size_t pi = 0;
+  for (int j = 0; j < nt; ++j) {
+    tc0[(size_t)j] = (int32_t)ci0.size();
+    for (; pi < pieces.size() && pieces[pi].trial == j; ++pi) {
+      const Piece &p = pieces[pi];
+      for (int64_t a = 0; a < p.len; a += CH) {
+        ci0.push_back(p.row0 + a);
+        cin.push_back(p.in0 + a);
+        clen.push_back((int32_t)std::min<int64_t>(CH, p.len - a));
+        ctr.push_back(j);
+      }
+    }
+  }
+  tc0[(size_t)nt] = (int32_t)ci0.size();
+  // per-chunk tables (small host-built plans, not per-pair data)
+  upload(g, S.chunk_i0, ci0.data(), ci0.size() * 8);
+  upload(g, S.in_base, cin.data(), cin.size() * 8);
+  upload(g, S.chunk_len, clen.data(), clen.size() * 4);
+  upload(g, S.chunk_trial, ctr.data(), ctr.size() * 4);
+  upload(g, S.trial_chunk0, tc0.data(), tc0.size() * 4);
+  return (int64_t)ci0.size();
+}
+
+// Group `nt` trials whose pairs are given as pieces into out.members /
+// out.head (and okeys) at the global positions seg_all[t0 + j].
+void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &pieces, int32_t t0,
+                  int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,
+                  const uint32_t *rowid, uint32_t val_base, Groups &out, uint64_t *okeys,
+                  GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter,
+                  int st_local) {
   int64_t maxseg = 0, npairs = 0;
   for (int j = 0; j < nt; ++j) {
     const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
@@ -329,46 +391,19 @@ void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, 
     npairs += L;
   }
   if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
-  // final buckets of ~2-4K pairs (the shared-memory sort holds 8K); the
+  // final buckets of ~1-2K pairs (the shared-memory sort holds 4K); the
   // coarse scatter fans out to <= 1024 buckets, a second level splits them
-  // further for very long trial segments; chunks of >= 64 pairs per bucket
+  // further for very long trial segments
   int32_t bits = 0, bits1 = 0;
   group_bits(maxseg, &bits, &bits1);
   const bool two = bits != bits1;
   const int64_t nbins = (int64_t)1 << bits;
   const int64_t nb1 = (int64_t)1 << bits1;
-  const int64_t CH = group_chunk_pairs();
-  (void)nb1;
-  std::vector<int64_t> ci0, inb((size_t)nt), seg((size_t)nt + 1);
-  std::vector<int32_t> clen, ctr, tc0((size_t)nt + 1);
-  for (int j = 0; j < nt; ++j) {
-    tc0[(size_t)j] = (int32_t)ci0.size();
-    inb[(size_t)j] = (int64_t)j * stride;
-    seg[(size_t)j] = seg_all[(size_t)t0 + j];
-    const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
-    for (int64_t a = 0; a < L; a += CH) {
-      ci0.push_back(a);
-      clen.push_back((int32_t)std::min<int64_t>(CH, L - a));
-      ctr.push_back(j);
-    }
-  }
-  seg[(size_t)nt] = seg_all[(size_t)t0 + nt];
-  tc0[(size_t)nt] = (int32_t)ci0.size();
-  const int64_t nch = (int64_t)ci0.size();
-  auto up = [&](DBuf &b, const void *h, size_t bytes) {
-    if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
-    if (bytes) CK(cudaMemcpyAsync(b.p, h, bytes, cudaMemcpyHostToDevice, g->stream));
-  };
-  auto need = [&](DBuf &b, size_t bytes) {
-    if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
-  };
-  // per-chunk tables (small host-built plans, not per-pair data)
-  up(S.chunk_i0, ci0.data(), ci0.size() * 8);
-  up(S.chunk_len, clen.data(), clen.size() * 4);
-  up(S.chunk_trial, ctr.data(), ctr.size() * 4);
-  up(S.in_base, inb.data(), inb.size() * 8);
-  up(S.seg, seg.data(), seg.size() * 8);
-  up(S.trial_chunk0, tc0.data(), tc0.size() * 4);
+  const int64_t nch = build_chunks(g, pieces, nt, S);
+  std::vector<int64_t> seg((size_t)nt + 1);
+  for (int j = 0; j <= nt; ++j) seg[(size_t)j] = seg_all[(size_t)t0 + j];
+  upload(g, S.seg, seg.data(), seg.size() * 8);
+  auto need = [&](DBuf &b, size_t bytes) { ::need(g, b, bytes); };
   need(S.counts, (size_t)(nch * nb1) * 4);
   need(S.bstart1, (size_t)(nt * nb1) * 4);
   need(S.bsize1, (size_t)(nt * nb1) * 4);
@@ -394,7 +429,7 @@ void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, 
   a.plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
   a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
   a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
-  a.plan.in_base = ptr<int64_t>(S.in_base);
+  a.plan.chunk_in0 = ptr<int64_t>(S.in_base);
   a.plan.seg = ptr<int64_t>(S.seg);
   a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
   a.keys = keys;
@@ -414,6 +449,7 @@ void group_chunk(sg_graph *g, const uint64_t *keys, int64_t stride, int32_t t0, 
   a.big_count = ptr<uint32_t>(S.big_count);
   a.members = ptr<uint32_t>(out.members);
   a.head = ptr<uint32_t>(out.head);
+  a.okeys = okeys;
   st_begin(g, st_hist);
   CK(group_hist(a, g->stream));
   CK(group_offsets(a, g->stream));
@@ -478,6 +514,194 @@ std::vector<uint64_t> recompute_ids(sg_graph *g, int level, const std::vector<in
   return out;
 }
 
+// ---------------------------------------------------------------- multi-rank
+[[noreturn]] void require_single(sg_graph *g, const std::string &what) {
+  fail(g, SG_EINVAL, what + " needs world == 1 (gather the per-rank groups with the getters)");
+}
+
+// Pass-II dense index k, identical for every world size: S1' nodes are ordered
+// by (pass-I trial j, key) and key ranges are ordered by rank, so the local
+// S1' rows of trial j (rows [first_j, first_{j+1})) get
+// k = K_j + sum_{r' < rank} S[j][r'] + (i - first_j).
+void assign_s1p_index(sg_graph *g, PassOut &P) {
+  Groups &G1 = g->grp[0];
+  const int c1 = G1.c, R = g->world, me = g->rank;
+  DBuf dseg, dcnt, dfirst, doff;
+  upload(g, dseg, G1.seg.data(), G1.seg.size() * 8);
+  dalloc(g, dcnt, (size_t)c1 * 8);
+  CK(cudaMemsetAsync(dcnt.p, 0, (size_t)c1 * 8, g->stream));
+  CK(rows_per_trial(ptr<int64_t>(P.rstart), P.nrows, ptr<int64_t>(dseg), c1,
+                    ptr<unsigned long long>(dcnt), g->stream));
+  std::vector<int64_t> cnt = d2h<int64_t>(g, dcnt, (size_t)c1);
+  std::vector<int64_t> all((size_t)c1 * R);
+  x_allgather_i64(g, cnt.data(), c1, all.data());
+  std::vector<int64_t> first((size_t)c1 + 1), off((size_t)c1);
+  int64_t K = 0;
+  sg_s1p_offsets(R, me, c1, all.data(), first.data(), off.data(), &K);
+  g->s1p_global = K;
+  g->s1p_k0 = -1;                       // the local k values are not one range
+  P.blocks = first;                     // rows grouped by pass-I trial
+  upload(g, dfirst, first.data(), first.size() * 8);
+  upload(g, doff, off.data(), off.size() * 8);
+  dalloc(g, P.rowid, (size_t)P.nrows * 4);
+  CK(assign_rowid(ptr<uint32_t>(P.rowid), P.nrows, ptr<int64_t>(dfirst), ptr<int64_t>(doff), c1,
+                  g->stream));
+  for (DBuf *b : {&dseg, &dcnt, &dfirst, &doff}) dfree(g, *b);
+}
+
+// Owner partition of one key chunk: pairs of (trial tl, row block b) go to
+// rank owner(key) = floor(key * R / 2^64) (contiguous key ranges, so the
+// canonical key order is rank-major).  Virtual trial vt = tl * nblk + b.
+// Phase `starts == nullptr`: counts only (mine[vt * R + d]).  Otherwise the
+// pairs are written dest-major (then vt, then row order) into skeys / svals.
+void owner_partition(sg_graph *g, PassOut &P, KeyChunk &ch, GroupScratch &S,
+                     std::vector<int64_t> *mine, const std::vector<int64_t> *starts,
+                     uint64_t *skeys, uint32_t *svals) {
+  const int R = g->world;
+  const std::vector<int64_t> &Bk = P.blocks;
+  const int nblk = (int)Bk.size() - 1;
+  const int nvt = ch.nt * nblk;
+  std::vector<Piece> pieces;
+  for (int tl = 0; tl < ch.nt; ++tl)
+    for (int b = 0; b < nblk; ++b)
+      if (Bk[(size_t)b + 1] > Bk[(size_t)b])
+        pieces.push_back(Piece{tl * nblk + b, (int64_t)tl * P.key_stride + Bk[(size_t)b],
+                               Bk[(size_t)b + 1] - Bk[(size_t)b], Bk[(size_t)b]});
+  const int64_t nch = build_chunks(g, pieces, nvt, S);
+  need(g, S.counts, (size_t)(nch * R) * 4);
+  need(g, S.bsize1, (size_t)nvt * R * 4);
+  need(g, S.bstart1, (size_t)nvt * R * 4);
+  GroupArgs a;
+  a.plan.c = nvt;
+  a.plan.nb1 = R;
+  a.plan.nbins = R;
+  a.plan.nchunks = nch;
+  a.plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
+  a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
+  a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
+  a.plan.chunk_in0 = ptr<int64_t>(S.in_base);
+  a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
+  a.keys = ptr<uint64_t>(ch.keys);
+  a.vals = nullptr;
+  a.rowid = ptr<uint32_t>(P.rowid);
+  a.val_base = 0;
+  a.counts = ptr<uint32_t>(S.counts);
+  a.bsize1 = ptr<uint32_t>(S.bsize1);
+  a.bstart1 = ptr<uint32_t>(S.bstart1);
+  CK(group_hist(a, g->stream));
+  CK(group_colscan(a, g->stream));
+  if (!starts) {
+    std::vector<uint32_t> bs = d2h<uint32_t>(g, S.bsize1, (size_t)nvt * R);
+    mine->assign(bs.begin(), bs.end());
+    return;
+  }
+  std::vector<uint32_t> st32(starts->begin(), starts->end());
+  upload(g, S.bstart1, st32.data(), st32.size() * 4);
+  std::vector<int64_t> zeros((size_t)nvt + 1, 0);
+  upload(g, S.seg, zeros.data(), zeros.size() * 8);
+  a.plan.seg = ptr<int64_t>(S.seg);
+  a.akeys = skeys;
+  a.avals = svals;
+  CK(group_scatter(a, g->num_sms, g->stream));
+}
+
+// Exchange + grouping of one level on a multi-rank handle.
+void group_multi(sg_graph *g, int level) {
+  PassOut &P = g->pass[level];
+  Groups &out = g->grp[level];
+  const int c = P.c, R = g->world, me = g->rank;
+  const int nblk = (int)P.blocks.size() - 1;
+  const int st_x = level == 0 ? kStX1 : kStX2;
+  GroupScratch S;
+  // phase 1: owner counts of every chunk, exchanged (all ranks: all chunks)
+  std::vector<std::vector<int64_t>> mine(P.chunks.size()), all(P.chunks.size());
+  for (size_t k = 0; k < P.chunks.size(); ++k) {
+    KeyChunk &ch = P.chunks[k];
+    if (!ch.computed) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+    st_begin(g, st_x);
+    owner_partition(g, P, ch, S, &mine[k], nullptr, nullptr, nullptr);
+    const int64_t n = (int64_t)ch.nt * nblk * R;
+    all[k].resize((size_t)n * R);
+    x_allgather_i64(g, mine[k].data(), n, all[k].data());
+    st_end(g, st_x);
+  }
+  // local trial segments of the received pairs
+  free_groups(g, out);
+  out.c = c;
+  out.seg.assign((size_t)c + 1, 0);
+  for (size_t k = 0; k < P.chunks.size(); ++k) {
+    const KeyChunk &ch = P.chunks[k];
+    const int64_t n = (int64_t)ch.nt * nblk * R;
+    for (int tl = 0; tl < ch.nt; ++tl) {
+      int64_t tot = 0;
+      for (int s = 0; s < R; ++s)
+        for (int b = 0; b < nblk; ++b) tot += all[k][(size_t)(s * n + ((int64_t)tl * nblk + b) * R + me)];
+      out.seg[(size_t)ch.t0 + tl + 1] = tot;
+    }
+  }
+  for (int j = 0; j < c; ++j) out.seg[(size_t)j + 1] += out.seg[(size_t)j];
+  out.npairs = out.seg[(size_t)c];
+  dalloc(g, out.members, (size_t)out.npairs * 4);
+  dalloc(g, out.okeys, (size_t)out.npairs * 8);
+  dalloc(g, out.head, (size_t)((out.npairs + 31) / 32) * 4);
+  CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
+  // phase 2: per chunk, partition to send buffers, all-to-all, group
+  for (size_t k = 0; k < P.chunks.size(); ++k) {
+    KeyChunk &ch = P.chunks[k];
+    const int nvt = ch.nt * nblk;
+    const int64_t n = (int64_t)nvt * R;
+    const std::vector<int64_t> &my = mine[k];
+    std::vector<int64_t> soff((size_t)R + 1, 0), starts((size_t)nvt * R);
+    for (int d = 0; d < R; ++d) {
+      int64_t run = soff[(size_t)d];
+      for (int vt = 0; vt < nvt; ++vt) {
+        starts[(size_t)vt * R + d] = run;
+        run += my[(size_t)vt * R + d];
+      }
+      soff[(size_t)d + 1] = run;
+    }
+    std::vector<int64_t> roff((size_t)R + 1, 0);
+    for (int s = 0; s < R; ++s) {
+      int64_t t = 0;
+      for (int vt = 0; vt < nvt; ++vt) t += all[k][(size_t)(s * n + (int64_t)vt * R + me)];
+      roff[(size_t)s + 1] = roff[(size_t)s] + t;
+    }
+    DBuf skeys, svals, rkeys, rvals;
+    dalloc(g, skeys, (size_t)soff[(size_t)R] * 8);
+    dalloc(g, svals, (size_t)soff[(size_t)R] * 4);
+    dalloc(g, rkeys, (size_t)roff[(size_t)R] * 8);
+    dalloc(g, rvals, (size_t)roff[(size_t)R] * 4);
+    st_begin(g, st_x);
+    owner_partition(g, P, ch, S, nullptr, &starts, ptr<uint64_t>(skeys), ptr<uint32_t>(svals));
+    dfree(g, ch.keys);
+    ch.computed = false;
+    x_alltoallv(g, skeys.p, soff.data(), rkeys.p, roff.data(), 8);
+    x_alltoallv(g, svals.p, soff.data(), rvals.p, roff.data(), 4);
+    st_end(g, st_x);
+    dfree(g, skeys);
+    dfree(g, svals);
+    // received pieces in canonical generator order: trial, row block, source
+    std::vector<Piece> pieces;
+    for (int tl = 0; tl < ch.nt; ++tl)
+      for (int b = 0; b < nblk; ++b)
+        for (int s = 0; s < R; ++s) {
+          const int vt = tl * nblk + b;
+          int64_t o = roff[(size_t)s];
+          for (int v2 = 0; v2 < vt; ++v2) o += all[k][(size_t)(s * n + (int64_t)v2 * R + me)];
+          const int64_t len = all[k][(size_t)(s * n + (int64_t)vt * R + me)];
+          if (len > 0) pieces.push_back(Piece{tl, o, len, 0});
+        }
+    group_pieces(g, ptr<uint64_t>(rkeys), pieces, ch.t0, ch.nt, out.seg, ptr<uint32_t>(rvals),
+                 nullptr, 0, out, ptr<uint64_t>(out.okeys), S, nullptr,
+                 level == 0 ? kStHist1 : kStHist2, level == 0 ? kStScatter1 : kStScatter2,
+                 level == 0 ? kStLocal1 : kStLocal2);
+    dfree(g, rkeys);
+    dfree(g, rvals);
+  }
+  free_scratch(g, S);
+  g->pairs_global[level] = exchange_sum(g, out.npairs);
+}
+
 // Host view of a grouped level: per-trial group ranges, group offsets, ids.
 struct HostGroups {
   std::vector<int64_t> trial_goffs, offs;
@@ -508,6 +732,13 @@ void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
   const int64_t G = (int64_t)H.offs.size();
   H.offs.push_back(q.npairs);
   if (!want_ids) return;
+  if (q.okeys.p) {
+    // multi-rank: the grouping kept the sorted keys; id = fmix^-1(key)
+    std::vector<uint64_t> ok = d2h<uint64_t>(g, q.okeys, (size_t)q.npairs);
+    H.ids.resize((size_t)G);
+    for (int64_t x = 0; x < G; ++x) H.ids[(size_t)x] = fmix_inv(ok[(size_t)H.offs[(size_t)x]]);
+    return;
+  }
   // id of a group = the shingle of its first (smallest) generator in that trial
   std::vector<uint32_t> rid;
   if (level == 0) rid = d2h<uint32_t>(g, p.rowid, (size_t)p.nrows);
@@ -547,6 +778,27 @@ sg_status sg_partition_rows(int64_t n, const int64_t *row_ptr, int32_t world, in
     bounds[r] = u;
   }
   bounds[world] = n;
+  return SG_OK;
+}
+
+sg_status sg_s1p_offsets(int32_t world, int32_t rank, int32_t c1, const int64_t *all,
+                         int64_t *first, int64_t *off, int64_t *total) {
+  if (world < 1 || rank < 0 || rank >= world || c1 < 0 || !all || !first || !off) return SG_EINVAL;
+  int64_t K = 0, f = 0;
+  for (int j = 0; j < c1; ++j) {
+    int64_t before = 0, sum = 0;
+    for (int r = 0; r < world; ++r) {
+      const int64_t v = all[(int64_t)r * c1 + j];
+      if (r < rank) before += v;
+      sum += v;
+    }
+    first[j] = f;
+    off[j] = K + before - f;
+    f += all[(int64_t)rank * c1 + j];
+    K += sum;
+  }
+  first[c1] = f;
+  if (total) *total = K;
   return SG_OK;
 }
 
@@ -735,12 +987,11 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     dfree(g, tot);
     P.nrows = nrows;
     P.key_stride = key_stride_for(nrows);
-    if (level == 0 && g->world > 1) {
-      exchange_row_counts(g, 0, nrows);  // n_e global
-    } else if (level == 0) {
-      g->n_e_global = nrows;
+    P.blocks = {0, nrows};
+    if (level == 0) {
+      g->n_e_global = g->world > 1 ? exchange_sum(g, nrows) : nrows;
     } else if (g->world > 1) {
-      exchange_row_counts(g, 1, nrows);  // |S1'| global, k0 (canonical dense index)
+      assign_s1p_index(g, P);            // |S1'| global, canonical dense index per row
     } else {
       g->s1p_global = nrows;
       g->s1p_k0 = 0;
@@ -755,7 +1006,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     st_end(g, st_all);
     sync(g);
     g->state = level == 0 ? kPassed1 : kPassed2;
-  });
+  }, true);
 }
 
 sg_status group_by_shingle(sg_graph *g) {
@@ -768,7 +1019,7 @@ sg_status group_by_shingle(sg_graph *g) {
     const int c = P.c;
     st_begin(g, level == 0 ? kStGroup1 : kStGroup2);
     if (g->world > 1) {
-      exchange_and_group(g, level);
+      group_multi(g, level);
     } else {
       Groups &out = g->grp[level];
       free_groups(g, out);
@@ -784,9 +1035,12 @@ sg_status group_by_shingle(sg_graph *g) {
       GroupScratch S;
       for (auto &ch : P.chunks) {
         if (!ch.computed) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
-        group_chunk(g, ptr<uint64_t>(ch.keys), P.key_stride, ch.t0, ch.nt, out.seg, nullptr, rowid,
-                    base, out, S, &ch.keys, level == 0 ? kStHist1 : kStHist2,
-                    level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2);
+        std::vector<Piece> pieces;
+        for (int tl = 0; tl < ch.nt; ++tl)
+          pieces.push_back(Piece{tl, (int64_t)tl * P.key_stride, P.nrows, 0});
+        group_pieces(g, ptr<uint64_t>(ch.keys), pieces, ch.t0, ch.nt, out.seg, nullptr, rowid, base,
+                     out, nullptr, S, &ch.keys, level == 0 ? kStHist1 : kStHist2,
+                     level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2);
         ch.computed = false;
       }
       free_scratch(g, S);
@@ -797,7 +1051,7 @@ sg_status group_by_shingle(sg_graph *g) {
     g->groups_global[level] = -1;  // computed lazily by sg_get_counts
     if (level == 1) g->e2_global = -1;
     g->state = level == 0 ? kGrouped1 : kGrouped2;
-  });
+  }, true);
 }
 
 sg_status shingle_graph_reset(sg_graph *g) {
@@ -825,7 +1079,7 @@ void shingle_graph_destroy(sg_graph *g) {
     PassOut &p = g->pass[l];
     for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) rel(b->p);
     for (auto &ch : p.chunks) rel(ch.keys.p);
-    for (DBuf *b : {&g->grp[l].members, &g->grp[l].head}) rel(b->p);
+    for (DBuf *b : {&g->grp[l].members, &g->grp[l].head, &g->grp[l].okeys}) rel(b->p);
   }
   for (DBuf *b : {&g->row_ptr, &g->col}) rel(b->p);
   for (auto &c : g->cache) rel(c.p);
@@ -879,7 +1133,7 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[16]) {
       counts[12 + l] = P.deferred ? -nch : nch;
     }
     counts[14] = counts[15] = 0;
-  });
+  }, true);
 }
 
 sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *rowid,
@@ -914,7 +1168,13 @@ sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *r
           sync(g);
         }
       } else {
-        for (int64_t r = 0; r < P.nrows; ++r) rowid[r] = (uint32_t)(g->s1p_k0 + r);
+        if (P.rowid.p && P.nrows) {           // multi-rank: canonical k of each row
+          CK(cudaMemcpyAsync(rowid, P.rowid.p, (size_t)P.nrows * 4, cudaMemcpyDeviceToHost,
+                             g->stream));
+          sync(g);
+        } else {
+          for (int64_t r = 0; r < P.nrows; ++r) rowid[r] = (uint32_t)(g->s1p_k0 + r);
+        }
       }
     }
   });
@@ -926,7 +1186,6 @@ sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64
     if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
     const int l = level - 1;
     if (g->state < (l == 0 ? kGrouped1 : kGrouped2)) fail(g, SG_ESTATE, "not grouped yet");
-    if (g->world > 1 && ids) exchange_require_single(g, "sg_get_groups ids");
     HostGroups H;
     host_groups(g, l, H, ids != nullptr);
     const int64_t G = (int64_t)H.offs.size() - 1;
@@ -1005,7 +1264,7 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
   return guarded(g, [&] {
     if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
     if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
-    if (g->world > 1) exchange_require_single(g, "report_dense_subgraphs");
+    if (g->world > 1) require_single(g, "report_dense_subgraphs");
     PassOut &P1 = g->pass[0];
     PassOut &P2 = g->pass[1];
     HostGroups H1, H2;

@@ -1,4 +1,13 @@
-// exchange.h — multi-GPU plumbing of libshingle.
+// exchange.h — multi-GPU transport of libshingle.
+//
+// Two backends behind one interface:
+//  * NCCL (one process per GPU; libnccl.so.2 is loaded with dlopen so the
+//    library also loads on machines without NCCL; the communicator is built
+//    from a 128-byte ncclUniqueId broadcast by the caller, e.g. through
+//    torch.distributed);
+//  * loopback (world virtual ranks inside one process, one host thread per
+//    rank, all on one device): collectives are host barriers + device
+//    memcpys.  It exercises the whole multi-rank path on a single GPU.
 #pragma once
 
 #include "sg_internal.cuh"
@@ -7,12 +16,19 @@ namespace sg {
 
 Exchange *exchange_create(sg_graph *g, const sg_dist *dist);
 void exchange_destroy(Exchange *x);
-// Pass rows: sums the local row count over ranks and sets the rank's base
-// (level 0: n_e and row base; level 1: |S1'| and the canonical k0).
-void exchange_row_counts(sg_graph *g, int level, int64_t local_rows);
-// Route the pass's pairs to their owner ranks and group them there.
-void exchange_and_group(sg_graph *g, int level);
+// A rank that fails inside a call marks the loopback group broken so its
+// peers leave their barriers with SG_ESTATE instead of waiting forever.
+void exchange_abort(Exchange *x);
+
+// all[r * n + i] = value i of rank r (host arrays).
+void x_allgather_i64(sg_graph *g, const int64_t *mine, int64_t n, int64_t *all);
 int64_t exchange_sum(sg_graph *g, int64_t v);
-void exchange_require_single(sg_graph *g, const char *what);
+int64_t exchange_min(sg_graph *g, int64_t v);
+// Device all-to-all-v: rank r sends send[soff[d] .. soff[d+1]) (elements of
+// eb bytes) to rank d and receives rank s's block into recv[roff[s] ..).
+// soff / roff are host arrays of world + 1 element offsets.  Enqueued on the
+// handle's stream; returns when the transfer has completed.
+void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
+                 const int64_t *roff, size_t eb);
 
 }  // namespace sg

@@ -64,10 +64,10 @@ struct GroupPlan {
   int64_t nchunks = 0;
   int64_t npairs = 0;
   // device tables
-  int64_t *chunk_i0 = nullptr;     // [nchunks] first pair of the chunk within its trial
+  int64_t *chunk_i0 = nullptr;     // [nchunks] row index of the chunk's first pair (implicit values)
   int32_t *chunk_len = nullptr;    // [nchunks]
   int32_t *chunk_trial = nullptr;  // [nchunks]
-  int64_t *in_base = nullptr;      // [c]   key index of pair 0 of trial j
+  int64_t *chunk_in0 = nullptr;    // [nchunks] key / explicit-value index of the chunk's first pair
   int64_t *seg = nullptr;          // [c+1] output position of pair 0 of trial j (global)
   int32_t *trial_chunk0 = nullptr; // [c+1] first chunk of each trial
 };
@@ -93,7 +93,16 @@ struct GroupArgs {
   // outputs
   uint32_t *members;           // [npairs]
   uint32_t *head;              // [(npairs+31)/32], zeroed by the launcher
+  uint64_t *okeys = nullptr;   // [npairs] sorted keys (optional; multi-rank getters)
 };
+
+// ---- multi-rank helpers (kernels_pass.cu) ----------------------------------
+// counts[j] = number of rows whose rstart lies in [seg[j], seg[j+1]) (zeroed by caller)
+cudaError_t rows_per_trial(const int64_t *rstart, int64_t nrows, const int64_t *seg, int32_t c,
+                           unsigned long long *counts, cudaStream_t st);
+// rowid[i] = i + off[j] for the trial j with first[j] <= i < first[j+1]
+cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, const int64_t *off,
+                         int32_t c, cudaStream_t st);
 
 int64_t group_local_capacity();
 int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
@@ -101,6 +110,7 @@ int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
 cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st);   // chunk prefixes + bsize1 only
 cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level plans only
 cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
@@ -110,7 +120,5 @@ cudaError_t group_big(const GroupArgs &g, uint32_t nbig, cudaStream_t st);
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);
 cudaError_t sum_i32(const int32_t *a, int64_t n, unsigned long long *d_out, cudaStream_t st);
-cudaError_t transpose_keys_to_ids(const uint64_t *keys, int64_t nrows, int32_t c, uint64_t *ids,
-                                  cudaStream_t st);
 
 }  // namespace sg

@@ -41,6 +41,12 @@ constexpr int kMaxBits = 15;         // final buckets per trial <= 32768
 constexpr int kMaxNb1 = 1 << kMaxSingleBits;
 constexpr int kMaxNb2 = 1 << (kMaxBits - kCoarseBits);
 
+// Coarse bin = floor(key * nb / 2^64): the top log2(nb) key bits when nb is a
+// power of two (buckets), contiguous key ranges for any nb (owner ranks).
+__device__ __forceinline__ uint32_t coarse_bin(uint64_t key, int64_t nb) {
+  return (uint32_t)__umul64hi(key, (uint64_t)nb);
+}
+
 __device__ __forceinline__ uint32_t val_at(const GroupArgs &g, int64_t in_idx, int64_t i) {
   if (g.vals) return g.vals[in_idx];
   if (g.rowid) return g.rowid[i];
@@ -132,12 +138,11 @@ __device__ __forceinline__ void stable_split(const uint64_t *sK, int len, int nb
 __global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ uint32_t hist[];
   const int64_t nb = g.plan.nb1;
-  const int bits = g.plan.bits1;
   for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) hist[i] = 0;
   __syncthreads();
   const int64_t k = blockIdx.x;
   const int j = g.plan.chunk_trial[k];
-  const uint64_t *__restrict__ keys = g.keys + g.plan.in_base[j] + g.plan.chunk_i0[k];
+  const uint64_t *__restrict__ keys = g.keys + g.plan.chunk_in0[k];
   const int len = g.plan.chunk_len[k];
   uint64_t kk[kChunk / kGThreads];
 #pragma unroll
@@ -147,7 +152,7 @@ __global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__
   }
 #pragma unroll
   for (int u = 0; u < kChunk / kGThreads; ++u)
-    if (threadIdx.x + u * kGThreads < len) atomicAdd(&hist[top_bits(kk[u], bits)], 1u);
+    if (threadIdx.x + u * kGThreads < len) atomicAdd(&hist[coarse_bin(kk[u], nb)], 1u);
   __syncthreads();
   uint32_t *out = g.counts + k * nb;
   for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) out[i] = hist[i];
@@ -202,11 +207,10 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
   extern __shared__ __align__(16) unsigned char smraw[];
   ScatterSmem &S = *reinterpret_cast<ScatterSmem *>(smraw);
   const int nb = (int)g.plan.nb1;
-  const int bits = g.plan.bits1;
   for (int64_t k = blockIdx.x; k < g.plan.nchunks; k += gridDim.x) {
     const int j = g.plan.chunk_trial[k];
     const int64_t i0 = g.plan.chunk_i0[k];
-    const int64_t in0 = g.plan.in_base[j] + i0;
+    const int64_t in0 = g.plan.chunk_in0[k];
     const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];   // scratch segment start
     const int len = g.plan.chunk_len[k];
     const uint32_t *pre = g.counts + k * nb;
@@ -226,7 +230,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
       }
     }
     __syncthreads();
-    stable_split(S.K, len, nb, [&](uint64_t key) { return top_bits(key, bits); }, S.cnt, S.sbst,
+    stable_split(S.K, len, nb, [&](uint64_t key) { return coarse_bin(key, nb); }, S.cnt, S.sbst,
                  S.ws, [&](int e, int p, uint32_t b) {
                    const int64_t o = sseg + S.gcur[b] + (p - (int)S.sbst[b]);
                    g.akeys[o] = S.K[e];
@@ -357,6 +361,13 @@ cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
   colscan_kernel<<<grid, 256, 0, st>>>(g);
   ++g_launches;
   binscan_kernel<<<(unsigned)g.plan.c, 1024, 0, st>>>(g);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st) {
+  dim3 grid((unsigned)((g.plan.nb1 + 255) / 256), (unsigned)g.plan.c);
+  colscan_kernel<<<grid, 256, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }

@@ -227,6 +227,7 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
       if (p < n) {
         const int e = pm[p];
         g.members[gbase + p] = S.V[e];
+        if (g.okeys) g.okeys[gbase + p] = K[e];
         head = (p == 0) || K[pm[p - 1]] != K[e];
       }
       const uint32_t hw = __ballot_sync(0xffffffffu, head);
@@ -265,7 +266,10 @@ __global__ void __launch_bounds__(1024) big_kernel(const __grid_constant__ Group
     }
   }
   const int64_t gbase = g.plan.seg[0] + sb;
-  for (int64_t p = threadIdx.x; p < n; p += blockDim.x) g.members[gbase + p] = V[p];
+  for (int64_t p = threadIdx.x; p < n; p += blockDim.x) {
+    g.members[gbase + p] = V[p];
+    if (g.okeys) g.okeys[gbase + p] = K[p];
+  }
   const int64_t w0 = gbase >> 5, w1 = (gbase + n - 1) >> 5;
   for (int64_t w = w0 + threadIdx.x; w <= w1; w += blockDim.x) {
     uint32_t bits = 0;

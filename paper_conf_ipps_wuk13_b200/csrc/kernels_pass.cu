@@ -157,6 +157,32 @@ __global__ void sel_grp_write_kernel(const uint32_t *__restrict__ head, int64_t 
   }
 }
 
+// ---- multi-rank helpers -------------------------------------------------------
+__device__ __forceinline__ int upper_trial(const int64_t *seg, int c, int64_t x) {
+  int lo = 0, hi = c;          // last j with seg[j] <= x
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (seg[mid] <= x) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void rows_per_trial_kernel(const int64_t *__restrict__ rstart, int64_t nrows,
+                                      const int64_t *__restrict__ seg, int c,
+                                      unsigned long long *counts) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nrows;
+       i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&counts[upper_trial(seg, c, rstart[i])], 1ull);
+}
+
+__global__ void assign_rowid_kernel(uint32_t *rowid, int64_t nrows, const int64_t *__restrict__ first,
+                                    const int64_t *__restrict__ off, int c) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nrows;
+       i += (int64_t)gridDim.x * blockDim.x)
+    rowid[i] = (uint32_t)(i + off[upper_trial(first, c, i)]);
+}
+
 }  // namespace
 
 int64_t sel_scratch_elems(int64_t items) { return (items + kSelPerBlock - 1) / kSelPerBlock + 1; }
@@ -211,5 +237,23 @@ cudaError_t select_groups_write(const uint32_t *head, int64_t npairs, int s, con
   return cudaGetLastError();
 }
 
+
+cudaError_t rows_per_trial(const int64_t *rstart, int64_t nrows, const int64_t *seg, int32_t c,
+                           unsigned long long *counts, cudaStream_t st) {
+  if (nrows == 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((nrows + 255) / 256, 148 * 8);
+  rows_per_trial_kernel<<<grid, 256, 0, st>>>(rstart, nrows, seg, c, counts);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, const int64_t *off,
+                         int32_t c, cudaStream_t st) {
+  if (nrows == 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((nrows + 255) / 256, 148 * 8);
+  assign_rowid_kernel<<<grid, 256, 0, st>>>(rowid, nrows, first, off, c);
+  ++g_launches;
+  return cudaGetLastError();
+}
 
 }  // namespace sg

@@ -96,6 +96,7 @@ struct PassOut {
   const uint32_t *entries = nullptr;  // row entries (pass I: col; pass II: G_I members)
   std::vector<KeyChunk> chunks; // trial chunks sized to the free HBM
   bool deferred = false;        // keys computed chunk by chunk inside group_by_shingle
+  std::vector<int64_t> blocks;  // row blocks in generator order (multi-rank exchange pieces)
 };
 
 // Grouped pairs of one level on this rank: per-trial segments of `members`
@@ -106,6 +107,7 @@ struct Groups {
   std::vector<int64_t> seg;            // [c+1] pair offsets per trial (host)
   DBuf members;                        // uint32 [npairs]
   DBuf head;                           // uint32 [(npairs + 31) / 32] head bits
+  DBuf okeys;                          // uint64 [npairs] sorted keys (multi-rank only)
 };
 
 constexpr int kNumStages = 16;
