@@ -106,6 +106,7 @@ cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, c
 
 int64_t group_local_capacity();
 int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
+int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
 // Bucket plan for trial segments of at most `maxseg` pairs.
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);

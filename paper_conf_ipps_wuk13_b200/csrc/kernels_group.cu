@@ -3,16 +3,15 @@
 // trial" (AMB-5).  The second half (sort inside a bucket + RLE)
 // is kernels_local.cu.  DESIGN.md §6.2.
 //
-//   1. hist     : per (trial, 8K-pair chunk) histogram of the top bits1 bits;
-//   2. offsets  : column prefix over chunks + per-trial bucket scan;
-//   3. scatter  : persistent, two 16-warp CTAs per SM.  A chunk's keys are
-//                 staged in shared memory, split into 16 contiguous warp
-//                 segments and ranked stably (__match_any_sync + per-warp
-//                 bucket counters); every pair is then written straight to its
-//                 bucket slot.  Fan-out <= 1024 buckets and <= 296 concurrent
-//                 chunks keep the partially written sectors (~19 MB) in L2;
-//   4. scatter2 : only for very long trial segments (two-level plans): one
-//                 CTA per coarse bucket splits it stably by the next <= 6 bits.
+//   1. hist     : per (trial, 4K-pair chunk) histogram of the coarse bin;
+//   2. offsets  : column prefix over the chunks of a trial (parallel over
+//                 chunk ranges) + per-trial bucket scan;
+//   3. scatter  : persistent, 16-warp CTAs.  A chunk is ranked stably in
+//                 registers (__match_any_sync + per-warp bin counters), placed
+//                 bucket-major in shared memory, then written out as
+//                 contiguous per-bucket runs (coalesced stores);
+//   4. scatter2 : two-level plans only: one CTA per coarse bucket splits it
+//                 stably by the next <= 7 bits with the same engine.
 // Stability matters: the input of every trial is in generator order, so the
 // members of one group (equal keys) arrive in ascending order and the local
 // sort never has to sort a group by member.
@@ -31,15 +30,15 @@ namespace {
 using grp::top_bits;
 
 constexpr int kGThreads = 512;
-constexpr int kSThreads = 512;       // 16 warps
-constexpr int kWarps = kSThreads / 32;
-constexpr int kChunk = 8192;         // pairs per scatter chunk (== hist chunk)
-constexpr int kPerLane = kChunk / kSThreads;   // 16
-constexpr int kMaxSingleBits = 10;   // single-level fan-out bound (<= 1024 buckets)
-constexpr int kCoarseBits = 9;       // two-level: first fan-out
-constexpr int kMaxBits = 15;         // final buckets per trial <= 32768
-constexpr int kMaxNb1 = 1 << kMaxSingleBits;
-constexpr int kMaxNb2 = 1 << (kMaxBits - kCoarseBits);
+constexpr int kSThreads = 512;                 // split kernels: 16 warps
+constexpr int kSWarps = kSThreads / 32;
+constexpr int kChunk = 4096;                   // pairs per chunk (hist and scatter)
+constexpr int kPerLane = kChunk / kSThreads;   // 8
+constexpr int kSeg = kChunk / kSWarps;         // 256 consecutive elements per warp
+constexpr int kMaxFan = 256;                   // bins of one split pass
+constexpr int kCoarseBits = 8;
+constexpr int kMaxBits = 15;                   // final buckets per trial <= 32768
+constexpr int kMaxFine = 1 << (kMaxBits - kCoarseBits);
 
 // Coarse bin = floor(key * nb / 2^64): the top log2(nb) key bits when nb is a
 // power of two (buckets), contiguous key ranges for any nb (owner ranks).
@@ -59,89 +58,113 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
-// ---- stable multi-split of the len <= kChunk keys staged in sK ---------------
-// Warp w owns the contiguous elements [w*512, w*512 + 512).  bin_of(k) in
-// [0, nb), nb <= 1024; cnt is uint16 [kWarps][nb]; sbst receives the bucket
-// starts within the chunk; emit(e, p, b) gets each element's chunk-relative
-// stable position p (bucket-major, input order inside a bucket).
-template <typename BIN, typename EMIT>
-__device__ __forceinline__ void stable_split(const uint64_t *sK, int len, int nb, BIN bin_of,
-                                             uint16_t *cnt, uint32_t *sbst, int64_t *ws,
-                                             EMIT emit) {
+// Element e of a chunk held by (warp w, lane, slot u): warps own contiguous
+// segments, so (w, u, lane) order is input order (stability).
+__device__ __forceinline__ int elem_of(int u) {
+  return (threadIdx.x >> 5) * kSeg + u * 32 + (threadIdx.x & 31);
+}
+
+struct SplitSmem {
+  uint64_t K[kChunk];                  // chunk, bucket-major after the split
+  uint32_t V[kChunk];
+  uint16_t cnt[kSWarps * kMaxFan];     // [warp][bin] running positions
+  uint32_t sbst[kMaxFan + 1];          // bin starts within the chunk
+  int64_t off[kMaxFan];                // output position - chunk position, per bin
+  int64_t gcur[kMaxFine];              // scatter2: running fine-bucket cursors
+  uint32_t tot[kMaxFine];              // scatter2: fine-bucket totals
+  int64_t ws[33];
+};
+
+// Rank the len <= kChunk pairs (kk, vv) of one chunk stably by bin_of(key) in
+// [0, nb) and place them bucket-major in S.K / S.V.  obase(b) gives the output
+// position of the first pair of bin b in this chunk; S.off[b] receives
+// obase(b) - (chunk position of that pair).  Ends with a barrier.
+template <typename BIN, typename OBASE>
+__device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
+                                            const uint64_t (&kk)[kPerLane],
+                                            const uint32_t (&vv)[kPerLane], BIN bin_of,
+                                            OBASE obase) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const uint32_t lt = lanemask_lt();
-  uint16_t *my = cnt + w * nb;
+  uint16_t *my = S.cnt + w * nb;
   for (int b = lane; b < nb; b += 32) my[b] = 0;
   __syncwarp();
   uint32_t pr[kPerLane];
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
-    const int e = w * (kPerLane * 32) + u * 32 + lane;
-    const bool valid = e < len;
+    const bool valid = elem_of(u) < len;
     const uint32_t vm = __ballot_sync(0xffffffffu, valid);
     pr[u] = 0;
     if (valid) {
-      const uint32_t b = bin_of(sK[e]);
+      const uint32_t b = bin_of(kk[u]);
       pr[u] = __match_any_sync(vm, b);
       if ((pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
     }
   }
   __syncthreads();
   {
-    // per bucket: exclusive prefix over the warps; bucket start = exclusive
-    // prefix over the buckets (thread t owns buckets [t*per, t*per + per))
-    const int per = (nb + blockDim.x - 1) / blockDim.x;   // <= 2
-    uint32_t tot[2] = {0, 0};
-    for (int y = 0; y < per; ++y) {
-      const int b = threadIdx.x * per + y;
-      if (b < nb) {
-        uint32_t run = 0;
-        for (int x = 0; x < kWarps; ++x) {
-          const uint32_t c = cnt[x * nb + b];
-          cnt[x * nb + b] = (uint16_t)run;
-          run += c;
-        }
-        tot[y] = run;
+    // bin-major, warp-minor exclusive prefix: thread t owns bin t (nb <= 256)
+    const int t = threadIdx.x;
+    uint32_t run = 0;
+    if (t < nb) {
+#pragma unroll 4
+      for (int x = 0; x < kSWarps; ++x) {
+        const uint32_t c = S.cnt[x * nb + t];
+        S.cnt[x * nb + t] = (uint16_t)run;
+        run += c;
       }
     }
     int64_t all;
-    int64_t ex = block_excl_scan<int64_t>((int64_t)tot[0] + tot[1], ws, &all);
-    for (int y = 0; y < per; ++y) {
-      const int b = threadIdx.x * per + y;
-      if (b < nb) {
-        sbst[b] = (uint32_t)ex;
-        for (int x = 0; x < kWarps; ++x) cnt[x * nb + b] += (uint16_t)ex;
-      }
-      ex += tot[y];
+    const int64_t ex = block_excl_scan<int64_t>((int64_t)run, S.ws, &all);
+    if (t < nb) {
+      S.sbst[t] = (uint32_t)ex;
+      S.off[t] = obase(t) - ex;
+#pragma unroll 4
+      for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + t] += (uint16_t)ex;
     }
+    if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
   __syncthreads();
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
-    const int e = w * (kPerLane * 32) + u * 32 + lane;
-    const bool valid = e < len;
+    const bool valid = elem_of(u) < len;
     const uint32_t vm = __ballot_sync(0xffffffffu, valid);
     if (valid) {
-      const uint32_t b = bin_of(sK[e]);
+      const uint32_t b = bin_of(kk[u]);
       const uint32_t rank = __popc(pr[u] & lt);
       const uint32_t base = my[b];
       __syncwarp(vm);
       if (rank == 0) my[b] = (uint16_t)(base + __popc(pr[u]));
       __syncwarp(vm);
-      emit(e, (int)(base + rank), b);
+      const uint32_t p = base + rank;
+      S.K[p] = kk[u];
+      S.V[p] = vv[u];
     }
   }
   __syncthreads();
 }
 
+// Write the placed chunk: consecutive threads take consecutive chunk
+// positions, which inside one bin are consecutive output positions.
+template <typename BIN>
+__device__ __forceinline__ void emit_runs(const SplitSmem &S, int len, BIN bin_of,
+                                          uint64_t *__restrict__ outK,
+                                          uint32_t *__restrict__ outV) {
+  for (int p = threadIdx.x; p < len; p += kSThreads) {
+    const uint64_t key = S.K[p];
+    const int64_t o = S.off[bin_of(key)] + p;
+    outK[o] = key;
+    outV[o] = S.V[p];
+  }
+}
+
 // ---- 1. histogram -----------------------------------------------------------
 __global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__ GroupArgs g) {
-  extern __shared__ uint32_t hist[];
+  __shared__ uint32_t hist[kMaxFan];
   const int64_t nb = g.plan.nb1;
   for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) hist[i] = 0;
   __syncthreads();
   const int64_t k = blockIdx.x;
-  const int j = g.plan.chunk_trial[k];
   const uint64_t *__restrict__ keys = g.keys + g.plan.chunk_in0[k];
   const int len = g.plan.chunk_len[k];
   uint64_t kk[kChunk / kGThreads];
@@ -160,20 +183,41 @@ __global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__
 
 // ---- 2. offsets ---------------------------------------------------------------
 // counts[k][b] <- exclusive prefix over the chunks of its trial; bsize1[j][b].
-__global__ void colscan_kernel(const __grid_constant__ GroupArgs g) {
+// Block (32 bins) x (32 chunk ranges): range sums, a scan over the ranges,
+// then each range rewrites its chunks.
+__global__ void __launch_bounds__(1024) colscan_kernel(const __grid_constant__ GroupArgs g) {
+  __shared__ uint32_t part[32][33];
   const int64_t nb = g.plan.nb1;
   const int j = blockIdx.y;
-  const int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (b >= nb) return;
+  const int bl = threadIdx.x & 31, pi = threadIdx.x >> 5;
+  const int64_t b = (int64_t)blockIdx.x * 32 + bl;
   const int k0 = g.plan.trial_chunk0[j], k1 = g.plan.trial_chunk0[j + 1];
-  uint32_t run = 0;
-  for (int k = k0; k < k1; ++k) {
-    uint32_t *p = g.counts + (int64_t)k * nb + b;
-    uint32_t v = *p;
-    *p = run;
-    run += v;
+  const int L = (k1 - k0 + 31) / 32;
+  const int a0 = k0 + pi * L, a1 = min(k1, a0 + L);
+  uint32_t s = 0;
+  if (b < nb)
+    for (int k = a0; k < a1; ++k) s += g.counts[(int64_t)k * nb + b];
+  part[pi][bl] = s;
+  __syncthreads();
+  if (pi == 0) {
+    uint32_t run = 0;
+    for (int x = 0; x < 32; ++x) {
+      const uint32_t v = part[x][bl];
+      part[x][bl] = run;
+      run += v;
+    }
+    if (b < nb) g.bsize1[(int64_t)j * nb + b] = run;
   }
-  g.bsize1[(int64_t)j * nb + b] = run;
+  __syncthreads();
+  if (b < nb) {
+    uint32_t run = part[pi][bl];
+    for (int k = a0; k < a1; ++k) {
+      uint32_t *p = g.counts + (int64_t)k * nb + b;
+      const uint32_t v = *p;
+      *p = run;
+      run += v;
+    }
+  }
 }
 
 // bstart1[j][b] = exclusive scan of bsize1[j][.] (relative to the segment).
@@ -194,64 +238,51 @@ __global__ void binscan_kernel(const __grid_constant__ GroupArgs g) {
   }
 }
 
-// ---- 3. stable coarse scatter (persistent, 2 CTAs / SM) -----------------------
-struct ScatterSmem {
-  uint64_t K[kChunk];
-  uint16_t cnt[kWarps * kMaxNb1];
-  uint32_t sbst[kMaxNb1];
-  uint32_t gcur[kMaxNb1];
-  int64_t ws[33];
-};
+// ---- 3. stable coarse scatter (persistent) ------------------------------------
+__device__ __forceinline__ void load_chunk(const GroupArgs &g, int64_t k, uint64_t (&kk)[kPerLane],
+                                           uint32_t (&vv)[kPerLane]) {
+  const int64_t i0 = g.plan.chunk_i0[k];
+  const int64_t in0 = g.plan.chunk_in0[k];
+  const int len = g.plan.chunk_len[k];
+#pragma unroll
+  for (int u = 0; u < kPerLane; ++u) {
+    const int e = elem_of(u);
+    if (e < len) {
+      kk[u] = g.keys[in0 + e];
+      vv[u] = val_at(g, in0 + e, i0 + e);
+    }
+  }
+}
 
 __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
-  ScatterSmem &S = *reinterpret_cast<ScatterSmem *>(smraw);
+  SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
   const int nb = (int)g.plan.nb1;
-  for (int64_t k = blockIdx.x; k < g.plan.nchunks; k += gridDim.x) {
+  auto bin = [&](uint64_t key) { return coarse_bin(key, nb); };
+  uint64_t kk[kPerLane];
+  uint32_t vv[kPerLane];
+  int64_t k = blockIdx.x;
+  if (k < g.plan.nchunks) load_chunk(g, k, kk, vv);
+  while (k < g.plan.nchunks) {
     const int j = g.plan.chunk_trial[k];
-    const int64_t i0 = g.plan.chunk_i0[k];
-    const int64_t in0 = g.plan.chunk_in0[k];
-    const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];   // scratch segment start
     const int len = g.plan.chunk_len[k];
-    const uint32_t *pre = g.counts + k * nb;
-    const uint32_t *bst = g.bstart1 + (int64_t)j * nb;
-    for (int b = threadIdx.x; b < nb; b += blockDim.x) S.gcur[b] = bst[b] + pre[b];
-    {
-      uint64_t kk[kPerLane];
-#pragma unroll
-      for (int u = 0; u < kPerLane; ++u) {
-        const int e = threadIdx.x + u * kSThreads;
-        if (e < len) kk[u] = g.keys[in0 + e];
-      }
-#pragma unroll
-      for (int u = 0; u < kPerLane; ++u) {
-        const int e = threadIdx.x + u * kSThreads;
-        if (e < len) S.K[e] = kk[u];
-      }
-    }
+    const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];   // scratch segment start
+    int64_t gb = 0;
+    if (threadIdx.x < nb)
+      gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
+    split_place(S, len, nb, kk, vv, bin, [&](int) { return gb; });
+    const int64_t kn = k + gridDim.x;
+    if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
+    emit_runs(S, len, bin, g.akeys, g.avals);
     __syncthreads();
-    stable_split(S.K, len, nb, [&](uint64_t key) { return coarse_bin(key, nb); }, S.cnt, S.sbst,
-                 S.ws, [&](int e, int p, uint32_t b) {
-                   const int64_t o = sseg + S.gcur[b] + (p - (int)S.sbst[b]);
-                   g.akeys[o] = S.K[e];
-                   g.avals[o] = val_at(g, in0 + e, i0 + e);
-                 });
+    k = kn;
   }
 }
 
 // ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
-struct Scatter2Smem {
-  uint64_t K[kChunk];
-  uint16_t cnt[kWarps * kMaxNb2];
-  uint32_t sbst[kMaxNb2];
-  uint32_t tot[kMaxNb2];
-  uint32_t gcur[kMaxNb2];
-  int64_t ws[33];
-};
-
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
-  Scatter2Smem &S = *reinterpret_cast<Scatter2Smem *>(smraw);
+  SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
   const int64_t q1 = blockIdx.x;                 // (trial, coarse bucket)
   const int64_t nb1 = g.plan.nb1;
   const int j = (int)(q1 / nb1);
@@ -279,36 +310,31 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
       const int64_t qf = (int64_t)j * g.plan.nbins + ((int64_t)b1 << bits2) + d;
       g.bstart[qf] = st1 + (uint32_t)ex;
       g.bsize[qf] = (uint32_t)v;
-      S.gcur[d] = st1 + (uint32_t)ex;
+      S.gcur[d] = sseg + st1 + ex;
     }
   }
   __syncthreads();
+  uint64_t kk[kPerLane];
+  uint32_t vv[kPerLane];
+  auto load = [&](int64_t c0) {
+    const int len = (int)min((int64_t)kChunk, n - c0);
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u) {
+      const int e = elem_of(u);
+      if (e < len) {
+        kk[u] = K[c0 + e];
+        vv[u] = V[c0 + e];
+      }
+    }
+  };
+  if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    {
-      uint64_t kk[kPerLane];
-#pragma unroll
-      for (int u = 0; u < kPerLane; ++u) {
-        const int e = threadIdx.x + u * kSThreads;
-        if (e < len) kk[u] = K[c0 + e];
-      }
-#pragma unroll
-      for (int u = 0; u < kPerLane; ++u) {
-        const int e = threadIdx.x + u * kSThreads;
-        if (e < len) S.K[e] = kk[u];
-      }
-    }
-    __syncthreads();
-    stable_split(S.K, len, nb2, fine, S.cnt, S.sbst, S.ws, [&](int e, int p, uint32_t d) {
-      const int64_t o = sseg + S.gcur[d] + (p - (int)S.sbst[d]);
-      g.bkeys[o] = S.K[e];
-      g.bvals[o] = V[c0 + e];
-    });
+    split_place(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    if (c0 + kChunk < n) load(c0 + kChunk);
+    emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts
-    for (int d = threadIdx.x; d < nb2; d += blockDim.x) {
-      const uint32_t end = d + 1 < nb2 ? S.sbst[d + 1] : (uint32_t)len;
-      S.gcur[d] += end - S.sbst[d];
-    }
+    for (int d = threadIdx.x; d < nb2; d += blockDim.x) S.gcur[d] += S.sbst[d + 1] - S.sbst[d];
     __syncthreads();
   }
 }
@@ -334,6 +360,7 @@ __global__ void sum_i32_kernel(const int32_t *__restrict__ a, int64_t n, unsigne
 }  // namespace
 
 int64_t group_chunk_pairs() { return kChunk; }
+int32_t group_max_fanout() { return kMaxFan; }
 
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1) {
   // final buckets of <= ~2K pairs on average (the shared-memory sort holds 4K)
@@ -345,41 +372,50 @@ void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1) {
   int b = 0;
   while ((maxseg >> b) > target && b < kMaxBits) ++b;
   *bits = b;
-  *bits1 = b <= kMaxSingleBits ? b : kCoarseBits;
+  *bits1 = std::min(b, kCoarseBits);
 }
 
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
-  const size_t smem = (size_t)g.plan.nb1 * sizeof(uint32_t);
-  hist_kernel<<<(unsigned)g.plan.nchunks, kGThreads, smem, st>>>(g);
-  ++g_launches;
-  return cudaGetLastError();
-}
-
-cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
-  dim3 grid((unsigned)((g.plan.nb1 + 255) / 256), (unsigned)g.plan.c);
-  colscan_kernel<<<grid, 256, 0, st>>>(g);
-  ++g_launches;
-  binscan_kernel<<<(unsigned)g.plan.c, 1024, 0, st>>>(g);
+  if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
+  hist_kernel<<<(unsigned)g.plan.nchunks, kGThreads, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
 
 cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st) {
-  dim3 grid((unsigned)((g.plan.nb1 + 255) / 256), (unsigned)g.plan.c);
-  colscan_kernel<<<grid, 256, 0, st>>>(g);
+  if (g.plan.c == 0) return cudaSuccess;
+  dim3 grid((unsigned)((g.plan.nb1 + 31) / 32), (unsigned)g.plan.c);
+  colscan_kernel<<<grid, 1024, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
 
+cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
+  cudaError_t e = group_colscan(g, st);
+  if (e != cudaSuccess || g.plan.c == 0) return e;
+  binscan_kernel<<<(unsigned)g.plan.c, 1024, 0, st>>>(g);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+static cudaError_t split_attr(const void *fn, int *per_sm) {
+  const size_t smem = sizeof(SplitSmem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, fn, kSThreads, smem);
+  *per_sm = std::max(*per_sm, 1);
+  return e;
+}
+
 cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
-  const size_t smem = sizeof(ScatterSmem);
-  cudaError_t e = cudaFuncSetAttribute(scatter_kernel,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
+  int per_sm = 1;
+  cudaError_t e = split_attr((const void *)scatter_kernel, &per_sm);
   if (e != cudaSuccess) return e;
-  const int grid = (int)std::min<int64_t>((int64_t)num_sms * 2, g.plan.nchunks);
-  scatter_kernel<<<grid, kSThreads, smem, st>>>(g);
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, g.plan.nchunks);
+  scatter_kernel<<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
@@ -387,11 +423,11 @@ cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
 cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   const int64_t nq1 = (int64_t)g.plan.c * g.plan.nb1;
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
-  const size_t smem = sizeof(Scatter2Smem);
-  cudaError_t e = cudaFuncSetAttribute(scatter2_kernel,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (g.plan.bits - g.plan.bits1 > kMaxBits - kCoarseBits) return cudaErrorInvalidValue;
+  int per_sm = 1;
+  cudaError_t e = split_attr((const void *)scatter2_kernel, &per_sm);
   if (e != cudaSuccess) return e;
-  scatter2_kernel<<<(unsigned)nq1, kSThreads, smem, st>>>(g);
+  scatter2_kernel<<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
