@@ -415,9 +415,9 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
     need(S.bkeys, (size_t)npairs * 8);
     need(S.bvals, (size_t)npairs * 4);
   }
-  need(S.big_list, (size_t)(nt * nbins) * 4);
-  need(S.big_count, 4);
-  CK(cudaMemsetAsync(S.big_count.p, 0, 4, g->stream));
+  need(S.big_list, (size_t)(nt * nbins) * 8);             // big + mid lists
+  need(S.big_count, 8);                                    // big + mid counts
+  CK(cudaMemsetAsync(S.big_count.p, 0, 8, g->stream));
   GroupArgs a;
   a.plan.c = nt;
   a.plan.bits = bits;
@@ -447,6 +447,8 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   a.bvals = two ? ptr<uint32_t>(S.bvals) : a.avals;
   a.big_list = ptr<uint32_t>(S.big_list);
   a.big_count = ptr<uint32_t>(S.big_count);
+  a.mid_list = a.big_list + nt * nbins;
+  a.mid_count = a.big_count + 1;
   a.members = ptr<uint32_t>(out.members);
   a.head = ptr<uint32_t>(out.head);
   a.okeys = okeys;
@@ -461,10 +463,6 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   st_end(g, st_scatter);
   st_begin(g, st_local);
   CK(group_local(a, g->num_sms, g->stream));
-  uint32_t nbig = 0;
-  CK(cudaMemcpyAsync(&nbig, S.big_count.p, 4, cudaMemcpyDeviceToHost, g->stream));
-  sync(g);
-  CK(group_big(a, nbig, g->stream));
   st_end(g, st_local);
 }
 

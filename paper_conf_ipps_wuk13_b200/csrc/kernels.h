@@ -88,8 +88,10 @@ struct GroupArgs {
   uint32_t *avals;
   uint64_t *bkeys;             // [npairs] final-bucketed pairs (== akeys if single-level)
   uint32_t *bvals;
-  uint32_t *big_list;          // [c*nbins] bucket ids with size > local capacity
-  uint32_t *big_count;         // [1]
+  uint32_t *big_list;          // [c*nbins] bucket ids with size > 4096 (global sort)
+  uint32_t *big_count;         // [1] (zeroed by the caller)
+  uint32_t *mid_list;          // [c*nbins] bucket ids with 1024 < size <= 4096 (CTA sort)
+  uint32_t *mid_count;         // [1] (zeroed by the caller)
   // outputs
   uint32_t *members;           // [npairs]
   uint32_t *head;              // [(npairs+31)/32], zeroed by the launcher
@@ -114,8 +116,9 @@ cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
 cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st);   // chunk prefixes + bsize1 only
 cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level plans only
+// Sort every final bucket and write members + head bits: warp tier, then the
+// mid and big tiers over the lists the warp tier filled (no host sync).
 cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
-cudaError_t group_big(const GroupArgs &g, uint32_t nbig, cudaStream_t st);
 
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,

@@ -11,7 +11,7 @@
 //                 bucket-major in shared memory, then written out as
 //                 contiguous per-bucket runs (coalesced stores);
 //   4. scatter2 : two-level plans only: one CTA per coarse bucket splits it
-//                 stably by the next <= 7 bits with the same engine.
+//                 stably by the next <= 8 bits with the same engine.
 // Stability matters: the input of every trial is in generator order, so the
 // members of one group (equal keys) arrive in ascending order and the local
 // sort never has to sort a group by member.
@@ -37,7 +37,7 @@ constexpr int kPerLane = kChunk / kSThreads;   // 8
 constexpr int kSeg = kChunk / kSWarps;         // 256 consecutive elements per warp
 constexpr int kMaxFan = 256;                   // bins of one split pass
 constexpr int kCoarseBits = 8;
-constexpr int kMaxBits = 15;                   // final buckets per trial <= 32768
+constexpr int kMaxBits = 16;                   // final buckets per trial <= 65536
 constexpr int kMaxFine = 1 << (kMaxBits - kCoarseBits);
 
 // Coarse bin = floor(key * nb / 2^64): the top log2(nb) key bits when nb is a
@@ -363,12 +363,12 @@ int64_t group_chunk_pairs() { return kChunk; }
 int32_t group_max_fanout() { return kMaxFan; }
 
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1) {
-  // final buckets of <= ~2K pairs on average (the shared-memory sort holds 4K)
+  // final buckets of 512-1024 pairs on average (the warp-tier sort holds 1K)
   // test hook SG_GROUP_TARGET: smaller target buckets (forces the two-level
   // partition and the big-bucket path on graphs the oracle can check)
   const char *e = getenv("SG_GROUP_TARGET");
-  int64_t target = e ? atoll(e) : 2048;
-  if (target <= 0) target = 2048;
+  int64_t target = e ? atoll(e) : 1024;
+  if (target <= 0) target = 1024;
   int b = 0;
   while ((maxseg >> b) > target && b < kMaxBits) ++b;
   *bits = b;

@@ -5,18 +5,21 @@
 // of one trial are still in generator order and a STABLE sort by key alone
 // yields the canonical (key, member) order.
 //
-// local_kernel: persistent CTAs of 8 warps (3 per SM overlap each other's
-// loads), one bucket of up to 4096 pairs at a time in shared memory:
-//   * two stable LSD multi-split passes on the 16 key bits after the bucket
-//     bits (8 bits each; warp segments, __match_any_sync ranks, a bin-major
-//     [digit][warp] counter matrix turned into starts by one block scan): the
-//     pairs of one group stay together and in member order;
-//   * the rare runs where distinct keys share those 16 bits out of order get
-//     a stable insertion sort by key;
-//   * members are written in sorted order (coalesced), one head bit per group
-//     start (ballot per 32 positions).
-// big_kernel: buckets above 4096 pairs, one CTA each, bitonic sort by the
-// total order (key, member) in global (L2-resident) memory.
+// Three tiers by bucket size n (mean ~600 pairs):
+//  * warp_local_kernel (n <= 1024): one warp per bucket, no block barriers.
+//    One sweep over the bucket's keys stores the 20 key bits after the
+//    bucket bits in the warp's shared-memory slice and builds both 10-bit
+//    digit histograms (packed 16-bit shared atomics); two stable placement
+//    passes (LSD; __match_any_sync peers, warp-private cursors) sort an index
+//    permutation; members are gathered through L1 and written in order
+//    (coalesced) with one head bit per group start.  The rare runs where
+//    distinct keys share the 20 bits out of order are detected while writing
+//    and get a stable insertion sort by key and a second write.  Larger
+//    buckets are appended to the mid / big lists.
+//  * local_kernel (n <= 4096, mid list): the same passes by a 256-thread CTA.
+//  * big_kernel (n > 4096, big list; groups of huge cliques): one CTA per
+//    bucket, bitonic sort by (key, member) in global (L2-resident) memory.
+// The mid and big tiers read their list lengths on the device (no host sync).
 #include <algorithm>
 
 #include "group_common.cuh"
@@ -31,12 +34,249 @@ namespace {
 using grp::bucket_extent;
 using grp::pair_less;
 
-constexpr int kLocalCap = 4096;
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+__device__ __forceinline__ void cp_async(void *sdst, const void *gsrc, int bytes) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(sdst);
+  if (bytes == 8) asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gsrc));
+  else asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gsrc));
+}
+
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.commit_group;\ncp.async.wait_all;\n" ::);
+}
+
+// Merge bucket-local head words hb[0, nw) (bit p = position p) into the
+// global head bit array at bit offset gbase; interior words are stored,
+// the two boundary words (shared with neighbouring buckets) are OR-ed.
+__device__ __forceinline__ void store_heads(uint32_t *head, const uint32_t *hb, int64_t gbase,
+                                            int n, int tid, int nthr) {
+  const int64_t w0 = gbase >> 5, w1 = (gbase + n - 1) >> 5;
+  const int off = (int)(gbase & 31);
+  const int nw = (n + 31) >> 5;
+  for (int64_t w = w0 + tid; w <= w1; w += nthr) {
+    const int k = (int)(w - w0);
+    uint32_t bits;
+    if (off == 0) {
+      bits = k < nw ? hb[k] : 0u;
+    } else {
+      const uint32_t lo = (k >= 1 && k - 1 < nw) ? hb[k - 1] : 0u;
+      const uint32_t hi = k < nw ? hb[k] : 0u;
+      bits = (lo >> (32 - off)) | (hi << off);
+    }
+    const int64_t lo_pos = w << 5, hi_pos = lo_pos + 32;
+    if (lo_pos >= gbase && hi_pos <= gbase + n) head[w] = bits;
+    else if (bits) atomicOr(&head[w], bits);
+  }
+}
+
+constexpr int kLocalCap = 4096;            // CTA tier capacity
+
+// ============================================================ warp tier
+constexpr int kWCap = 1024;
+constexpr int kWBatch = kWCap / 32;        // 32 batches of 32 positions
+constexpr int kWWarps = 7;                 // warps per CTA (3 CTAs, 21 warps per SM)
+constexpr int kWDigitBits = 10;            // two LSD passes = 20 key bits
+constexpr int kWDigits = 1 << kWDigitBits;
+
+struct __align__(16) WarpSmem {
+  uint32_t d20[kWCap];        // the 20 key bits after the bucket bits
+  uint16_t pa[kWCap];         // order after the first pass
+  uint16_t cA[kWDigits];      // low-digit counts -> cursors; then the final order
+  uint16_t cB[kWDigits];      // high-digit counts -> cursors
+  uint32_t hb[kWBatch];
+};
+
+// Exclusive scan in place of 1024 uint16 counters (lane owns 32 consecutive).
+__device__ __forceinline__ void warp_scan_1024(uint16_t *cnt) {
+  const int lane = threadIdx.x & 31;
+  uint32_t *w32 = reinterpret_cast<uint32_t *>(cnt) + lane * 16;
+  uint32_t v[16];
+  uint32_t s = 0;
+#pragma unroll
+  for (int x = 0; x < 16; ++x) {
+    v[x] = w32[x];
+    s += (v[x] & 0xFFFFu) + (v[x] >> 16);
+  }
+  uint32_t run = warp_incl_scan(s) - s;
+#pragma unroll
+  for (int x = 0; x < 16; ++x) {
+    const uint32_t lo = run;
+    const uint32_t hi = run + (v[x] & 0xFFFFu);
+    run = hi + (v[x] >> 16);
+    w32[x] = lo | (hi << 16);
+  }
+}
+
+// Stable placement pass: position of element e (visited in the order src,
+// identity if FIRST) = cursor[digit] + rank among same-digit peers of its
+// batch (__match_any_sync); the lowest peer advances the cursor.
+template <bool FIRST>
+__device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint16_t *src,
+                                           uint16_t *cur, uint16_t *dst, int shift) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  for (int i0 = 0; i0 < n; i0 += 32) {
+    const int i = i0 + lane;
+    const bool valid = i < n;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    if (valid) {
+      const uint16_t e = FIRST ? (uint16_t)i : src[i];
+      const uint32_t d = (S.d20[e] >> shift) & (kWDigits - 1);
+      const uint32_t m = __match_any_sync(vm, d);
+      const uint32_t rank = __popc(m & lt);
+      const uint32_t base = cur[d];
+      __syncwarp(vm);
+      if (rank == 0) cur[d] = (uint16_t)(base + __popc(m));
+      __syncwarp(vm);
+      dst[base + rank] = e;
+    }
+    __syncwarp();
+  }
+}
+
+// Write members (and sorted keys) in the order pm; head bits into S.hb.
+// Returns true if some adjacent pair is out of key order (a 20-bit tie).
+__device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n,
+                                          const uint16_t *pm, const uint64_t *Kg,
+                                          const uint32_t *Vg, int64_t gbase) {
+  const int lane = threadIdx.x & 31;
+  bool bad = false;
+  uint64_t carry = 0;
+  for (int p0 = 0; p0 < n; p0 += 32) {
+    const int p = p0 + lane;
+    const bool valid = p < n;
+    const int e = valid ? pm[p] : 0;
+    const uint64_t ke = valid ? Kg[e] : ~0ull;
+    const uint32_t ve = valid ? Vg[e] : 0u;
+    uint64_t prev = __shfl_up_sync(0xffffffffu, ke, 1);
+    if (lane == 0) prev = carry;
+    carry = __shfl_sync(0xffffffffu, ke, 31);
+    bool head = false;
+    if (valid) {
+      g.members[gbase + p] = ve;
+      if (g.okeys) g.okeys[gbase + p] = ke;
+      head = (p == 0) || prev != ke;
+      bad |= (p > 0) && ke < prev;
+    }
+    const uint32_t hw = __ballot_sync(0xffffffffu, head);
+    if (lane == 0) S.hb[p0 >> 5] = hw;
+  }
+  return __any_sync(0xffffffffu, bad);
+}
+
+__global__ void __launch_bounds__(kWWarps * 32) warp_local_kernel(const __grid_constant__ GroupArgs g) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  WarpSmem &S = reinterpret_cast<WarpSmem *>(smraw)[wl];
+  const int64_t nq = (int64_t)g.plan.c * g.plan.nbins;
+  const int bits = g.plan.bits;
+  const int64_t obase = g.plan.seg[0];     // scratch -> output position
+  const int64_t nwarps = (int64_t)gridDim.x * kWWarps;
+  for (int64_t q = (int64_t)blockIdx.x * kWWarps + wl; q < nq; q += nwarps) {
+    int64_t sb, n64;
+    bucket_extent(g, q, sb, n64);
+    if (n64 == 0) continue;
+    if (n64 > kWCap) {
+      if (lane == 0) {
+        if (n64 > kLocalCap) g.big_list[atomicAdd(g.big_count, 1u)] = (uint32_t)q;
+        else g.mid_list[atomicAdd(g.mid_count, 1u)] = (uint32_t)q;
+      }
+      continue;
+    }
+    const int n = (int)n64;
+    const uint64_t *Kg = g.bkeys + sb;
+    const uint32_t *Vg = g.bvals + sb;
+    {
+      uint4 *a4 = reinterpret_cast<uint4 *>(S.cA);
+      uint4 *b4 = reinterpret_cast<uint4 *>(S.cB);
+#pragma unroll
+      for (int x = 0; x < kWDigits / 256; ++x) {
+        a4[lane + 32 * x] = make_uint4(0, 0, 0, 0);
+        b4[lane + 32 * x] = make_uint4(0, 0, 0, 0);
+      }
+    }
+    __syncwarp();
+    // one sweep: the 20 sort bits of each key and both digit histograms
+    // (packed 16-bit counters, order-free); the values are prefetched into L1
+    for (int i0 = 0; i0 < n; i0 += 128) {
+      uint64_t k4[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int i = i0 + u * 32 + lane;
+        k4[u] = i < n ? Kg[i] : 0ull;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int i = i0 + u * 32 + lane;
+        if (i < n) {
+          const uint32_t d20 = (uint32_t)((k4[u] << bits) >> 44);
+          S.d20[i] = d20;
+          const uint32_t dl = d20 & (kWDigits - 1), dh = d20 >> kWDigitBits;
+          atomicAdd(reinterpret_cast<uint32_t *>(S.cA) + (dl >> 1), 1u << (16 * (dl & 1)));
+          atomicAdd(reinterpret_cast<uint32_t *>(S.cB) + (dh >> 1), 1u << (16 * (dh & 1)));
+          asm volatile("prefetch.global.L1 [%0];" ::"l"(Vg + i));
+        }
+      }
+    }
+    __syncwarp();
+    warp_scan_1024(S.cA);
+    warp_scan_1024(S.cB);
+    __syncwarp();
+    warp_place<true>(S, n, nullptr, S.cA, S.pa, 0);
+    uint16_t *pm = S.cA;                    // the low-digit cursors are spent
+    warp_place<false>(S, n, S.pa, S.cB, pm, kWDigitBits);
+    const int64_t gbase = obase + sb;
+    if (warp_emit(g, S, n, pm, Kg, Vg, gbase)) {
+      // distinct keys sharing the 20 bits out of key order: mark the start of
+      // each such equal-20-bit run, sort each run by key (stable), emit again
+      __syncwarp();
+      S.hb[lane] = 0;
+      __syncwarp();
+      for (int p = lane + 1; p < n; p += 32) {
+        const uint64_t kp = Kg[pm[p]];
+        if (kp < Kg[pm[p - 1]]) {
+          const uint32_t dp = S.d20[pm[p]];
+          int a = p - 1;
+          while (a > 0 && S.d20[pm[a - 1]] == dp) --a;
+          atomicOr(&S.hb[a >> 5], 1u << (a & 31));
+        }
+      }
+      __syncwarp();
+      uint32_t word = S.hb[lane];
+      __syncwarp();
+      while (word) {
+        const int a = lane * 32 + __ffs(word) - 1;
+        word &= word - 1;
+        const uint32_t da = S.d20[pm[a]];
+        int b = a + 1;
+        while (b < n && S.d20[pm[b]] == da) ++b;
+        for (int x = a + 1; x < b; ++x) {
+          const uint16_t e = pm[x];
+          const uint64_t ke = Kg[e];
+          int y = x - 1;
+          while (y >= a && ke < Kg[pm[y]]) { pm[y + 1] = pm[y]; --y; }   // strict: stable
+          pm[y + 1] = e;
+        }
+      }
+      __syncwarp();
+      warp_emit(g, S, n, pm, Kg, Vg, gbase);
+    }
+    __syncwarp();
+    store_heads(g.head, S.hb, gbase, n, lane, 32);
+    __syncwarp();
+  }
+}
+
+// ============================================================ CTA tier
 constexpr int kLThreads = 256;
 constexpr int kLWarps = kLThreads / 32;
 constexpr int kPerLane = kLocalCap / kLThreads;   // 16
-constexpr int kDigitBits = 8;                     // two stable LSD passes = 16 key bits
-constexpr int kDigits = 1 << kDigitBits;
+constexpr int kDigits = 256;
 constexpr int kCntPerThread = kDigits * kLWarps / kLThreads;   // 8
 
 struct LocalSmem {
@@ -51,12 +291,6 @@ struct LocalSmem {
   int64_t ws[33];
 };
 static_assert(kCntPerThread == 8, "counter scan assumes 8 per thread");
-
-__device__ __forceinline__ uint32_t lanemask_lt() {
-  uint32_t m;
-  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
-  return m;
-}
 
 // One stable multi-split pass over n <= 4096 elements: warp w owns the
 // positions [w*seg, (w+1)*seg) of the current order src (identity if null)
@@ -80,6 +314,7 @@ __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *sr
       pr[pos - seg_lo] = m;
       if ((m & lt) == 0) S.cnt[dg * kLWarps + w] += (uint16_t)__popc(m);
     }
+    __syncwarp();
   }
   __syncthreads();
   {
@@ -114,56 +349,28 @@ __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *sr
       __syncwarp(vm);
       dst[base + rank] = el;
     }
+    __syncwarp();
   }
   __syncthreads();
-}
-
-// Head-bit words of output positions [gbase, gbase + n) from the bucket-local
-// bit array hb (bit p = position p).
-__device__ __forceinline__ void store_heads(uint32_t *head, const uint32_t *hb, int64_t gbase,
-                                            int n) {
-  const int64_t w0 = gbase >> 5, w1 = (gbase + n - 1) >> 5;
-  const int off = (int)(gbase & 31);
-  const int nw = (n + 31) >> 5;
-  for (int64_t w = w0 + threadIdx.x; w <= w1; w += blockDim.x) {
-    const int k = (int)(w - w0);
-    uint32_t bits;
-    if (off == 0) {
-      bits = k < nw ? hb[k] : 0u;
-    } else {
-      const uint32_t lo = (k >= 1 && k - 1 < nw) ? hb[k - 1] : 0u;
-      const uint32_t hi = k < nw ? hb[k] : 0u;
-      bits = (lo >> (32 - off)) | (hi << off);
-    }
-    const int64_t lo_pos = w << 5, hi_pos = lo_pos + 32;
-    if (lo_pos >= gbase && hi_pos <= gbase + n) head[w] = bits;
-    else if (bits) atomicOr(&head[w], bits);
-  }
 }
 
 __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   LocalSmem &S = *reinterpret_cast<LocalSmem *>(smraw);
-  const int64_t nq = (int64_t)g.plan.c * g.plan.nbins;
   const int bits = g.plan.bits;
   const int64_t obase = g.plan.seg[0];     // scratch -> output position
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  for (int64_t q = blockIdx.x; q < nq; q += gridDim.x) {
+  const uint32_t nmid = *g.mid_count;
+  for (uint32_t li = blockIdx.x; li < nmid; li += gridDim.x) {
+    const int64_t q = g.mid_list[li];
     int64_t sb, n64;
     bucket_extent(g, q, sb, n64);
-    if (n64 == 0) continue;
-    if (n64 > kLocalCap) {
-      if (threadIdx.x == 0) g.big_list[atomicAdd(g.big_count, 1u)] = (uint32_t)q;
-      continue;
-    }
     const int n = (int)n64;
     for (int i = threadIdx.x; i < n; i += kLThreads) {
-      const unsigned sk = (unsigned)__cvta_generic_to_shared(&S.K[i]);
-      const unsigned sv = (unsigned)__cvta_generic_to_shared(&S.V[i]);
-      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sk), "l"(g.bkeys + sb + i));
-      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sv), "l"(g.bvals + sb + i));
+      cp_async(&S.K[i], g.bkeys + sb + i, 8);
+      cp_async(&S.V[i], g.bvals + sb + i, 4);
     }
-    asm volatile("cp.async.commit_group;\ncp.async.wait_all;\n" ::);
+    cp_async_wait_all();
     // (lsd_pass begins with a barrier after zeroing its counters)
     lsd_pass(S, n, nullptr, S.perm[0],
              [&](uint64_t key) { return (uint32_t)((key << (bits + 8)) >> 56); });
@@ -234,52 +441,56 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
       if (lane == 0) S.hb[p0 >> 5] = hw;
     }
     __syncthreads();
-    store_heads(g.head, S.hb, gbase, n);
+    store_heads(g.head, S.hb, gbase, n, threadIdx.x, blockDim.x);
     __syncthreads();
   }
 }
 
-// ---- big buckets: one CTA, bitonic in global memory ---------------------------
+// ============================================================ big tier
 __global__ void __launch_bounds__(1024) big_kernel(const __grid_constant__ GroupArgs g) {
-  const int64_t q = g.big_list[blockIdx.x];
-  int64_t sb, n;
-  bucket_extent(g, q, sb, n);
-  uint64_t *K = g.bkeys + sb;
-  uint32_t *V = g.bvals + sb;
-  int64_t M = 1;
-  while (M < n) M <<= 1;
-  for (int64_t k = 2; k <= M; k <<= 1) {
-    for (int64_t jj = k >> 1; jj > 0; jj >>= 1) {
-      for (int64_t t = threadIdx.x; t < (M >> 1); t += blockDim.x) {
-        const int64_t i = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
-        const int64_t l = (jj == (k >> 1)) ? (i ^ (k - 1)) : (i + jj);
-        if (l < n) {
-          const uint64_t ka = K[i], kb = K[l];
-          const uint32_t va = V[i], vb = V[l];
-          if (pair_less(kb, vb, ka, va)) {
-            K[i] = kb; K[l] = ka;
-            V[i] = vb; V[l] = va;
+  const uint32_t nbig = *g.big_count;
+  for (uint32_t li = blockIdx.x; li < nbig; li += gridDim.x) {
+    const int64_t q = g.big_list[li];
+    int64_t sb, n;
+    bucket_extent(g, q, sb, n);
+    uint64_t *K = g.bkeys + sb;
+    uint32_t *V = g.bvals + sb;
+    int64_t M = 1;
+    while (M < n) M <<= 1;
+    for (int64_t k = 2; k <= M; k <<= 1) {
+      for (int64_t jj = k >> 1; jj > 0; jj >>= 1) {
+        for (int64_t t = threadIdx.x; t < (M >> 1); t += blockDim.x) {
+          const int64_t i = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
+          const int64_t l = (jj == (k >> 1)) ? (i ^ (k - 1)) : (i + jj);
+          if (l < n) {
+            const uint64_t ka = K[i], kb = K[l];
+            const uint32_t va = V[i], vb = V[l];
+            if (pair_less(kb, vb, ka, va)) {
+              K[i] = kb; K[l] = ka;
+              V[i] = vb; V[l] = va;
+            }
           }
         }
+        __syncthreads();
       }
-      __syncthreads();
     }
-  }
-  const int64_t gbase = g.plan.seg[0] + sb;
-  for (int64_t p = threadIdx.x; p < n; p += blockDim.x) {
-    g.members[gbase + p] = V[p];
-    if (g.okeys) g.okeys[gbase + p] = K[p];
-  }
-  const int64_t w0 = gbase >> 5, w1 = (gbase + n - 1) >> 5;
-  for (int64_t w = w0 + threadIdx.x; w <= w1; w += blockDim.x) {
-    uint32_t bits = 0;
-    const int64_t lo = max(gbase, w << 5), hi = min(gbase + n, (w << 5) + 32);
-    for (int64_t gp = lo; gp < hi; ++gp) {
-      const int64_t p = gp - gbase;
-      if (p == 0 || K[p] != K[p - 1]) bits |= 1u << (gp & 31);
+    const int64_t gbase = g.plan.seg[0] + sb;
+    for (int64_t p = threadIdx.x; p < n; p += blockDim.x) {
+      g.members[gbase + p] = V[p];
+      if (g.okeys) g.okeys[gbase + p] = K[p];
     }
-    if (lo == (w << 5) && hi == (w << 5) + 32) g.head[w] = bits;
-    else if (bits) atomicOr(&g.head[w], bits);
+    const int64_t w0 = gbase >> 5, w1 = (gbase + n - 1) >> 5;
+    for (int64_t w = w0 + threadIdx.x; w <= w1; w += blockDim.x) {
+      uint32_t bits = 0;
+      const int64_t lo = max(gbase, w << 5), hi = min(gbase + n, (w << 5) + 32);
+      for (int64_t gp = lo; gp < hi; ++gp) {
+        const int64_t p = gp - gbase;
+        if (p == 0 || K[p] != K[p - 1]) bits |= 1u << (gp & 31);
+      }
+      if (lo == (w << 5) && hi == (w << 5) + 32) g.head[w] = bits;
+      else if (bits) atomicOr(&g.head[w], bits);
+    }
+    __syncthreads();
   }
 }
 
@@ -290,23 +501,34 @@ int64_t group_local_capacity() { return kLocalCap; }
 cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   const int64_t nq = (int64_t)g.plan.c * g.plan.nbins;
   if (nq == 0) return cudaSuccess;
-  const size_t smem = sizeof(LocalSmem);
-  cudaError_t e = cudaFuncSetAttribute(local_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem);
-  if (e != cudaSuccess) return e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_kernel, kLThreads, smem);
-  if (e != cudaSuccess) return e;
-  per_sm = std::max(per_sm, 1);
-  const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, nq);
-  local_kernel<<<grid, kLThreads, smem, st>>>(g);
-  ++g_launches;
-  return cudaGetLastError();
-}
-
-cudaError_t group_big(const GroupArgs &g, uint32_t nbig, cudaStream_t st) {
-  if (nbig == 0) return cudaSuccess;
-  big_kernel<<<nbig, 1024, 0, st>>>(g);
+  // warp tier over all buckets
+  {
+    const size_t smem = sizeof(WarpSmem) * kWWarps;
+    cudaError_t e = cudaFuncSetAttribute(warp_local_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, warp_local_kernel, kWWarps * 32, smem);
+    if (e != cudaSuccess) return e;
+    per_sm = std::max(per_sm, 1);
+    const int64_t want = (nq + kWWarps - 1) / kWWarps;
+    const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, want);
+    warp_local_kernel<<<grid, kWWarps * 32, smem, st>>>(g);
+    ++g_launches;
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  // CTA tier over the mid list (length read on the device)
+  {
+    const size_t smem = sizeof(LocalSmem);
+    cudaError_t e = cudaFuncSetAttribute(local_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+    local_kernel<<<num_sms * 2, kLThreads, smem, st>>>(g);
+    ++g_launches;
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  // big tier (length read on the device)
+  big_kernel<<<num_sms, 1024, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
