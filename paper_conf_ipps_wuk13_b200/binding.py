@@ -14,7 +14,8 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libshingle.so")
+# SG_LIB: test / A-B hook to load another build of the same library
+LIB_PATH = os.environ.get("SG_LIB") or os.path.join(_HERE, "libshingle.so")
 
 SG_OK, SG_EINVAL, SG_ENOMEM, SG_ESTATE, SG_ECUDA, SG_ENCCL, SG_EOVERFLOW = range(7)
 SG_DEVICE_PTRS = 0x1

@@ -314,12 +314,14 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
 
 // ---------------------------------------------------------------- grouping
 struct GroupScratch {
-  DBuf chunk_i0, chunk_len, chunk_trial, in_base, seg, trial_chunk0;
+  DBuf p_trial, p_in0, p_len, p_row0, p_chunk0, seg, trial_chunk0;
+  DBuf chunk_i0, chunk_in0, chunk_len, chunk_trial;
   DBuf counts, bstart1, bsize1, bstart, bsize, akeys, avals, bkeys, bvals, big_list, big_count;
 };
 
 void free_scratch(sg_graph *g, GroupScratch &S) {
-  for (DBuf *b : {&S.chunk_i0, &S.chunk_len, &S.chunk_trial, &S.in_base, &S.seg, &S.trial_chunk0,
+  for (DBuf *b : {&S.p_trial, &S.p_in0, &S.p_len, &S.p_row0, &S.p_chunk0, &S.seg, &S.trial_chunk0,
+                  &S.chunk_i0, &S.chunk_in0, &S.chunk_len, &S.chunk_trial,
                   &S.counts, &S.bstart1, &S.bsize1, &S.bstart, &S.bsize, &S.akeys, &S.avals,
                   &S.bkeys, &S.bvals, &S.big_list, &S.big_count})
     dfree(g, *b);
@@ -348,33 +350,51 @@ void need(sg_graph *g, DBuf &b, size_t bytes) {
   if (b.bytes < std::max<size_t>(bytes, 16)) dalloc(g, b, bytes);
 }
 
-// Chunk table of a partition over `nt` trials: pieces (ordered by trial, then
-// input order) cut into chunks of <= group_chunk_pairs() pairs.
-int64_t build_chunks(sg_graph *g, const std::vector<Piece> &pieces, int32_t nt, GroupScratch &S) {
+// Piece table of a partition over `nt` trials (pieces ordered by trial, then
+// input order; chunks of <= group_chunk_pairs() pairs are found on the device
+// by binary search over the pieces' first chunks).  Returns the chunk count.
+int64_t build_pieces(sg_graph *g, const std::vector<Piece> &pieces, int32_t nt, GroupScratch &S,
+                     GroupPlan &plan) {
   const int64_t CH = group_chunk_pairs();
-  std::vector<int64_t> ci0, cin;
-  std::vector<int32_t> clen, ctr, tc0((size_t)nt + 1, 0);
+  std::vector<int32_t> tr, tc0((size_t)nt + 1, 0);
+  std::vector<int64_t> in0, len, row0, c0;
+  int64_t nch = 0;
   size_t pi = 0;
   for (int j = 0; j < nt; ++j) {
-    tc0[(size_t)j] = (int32_t)ci0.size();
+    tc0[(size_t)j] = (int32_t)nch;
     for (; pi < pieces.size() && pieces[pi].trial == j; ++pi) {
       const Piece &p = pieces[pi];
-      for (int64_t a = 0; a < p.len; a += CH) {
-        ci0.push_back(p.row0 + a);
-        cin.push_back(p.in0 + a);
-        clen.push_back((int32_t)std::min<int64_t>(CH, p.len - a));
-        ctr.push_back(j);
-      }
+      if (p.len <= 0) continue;
+      tr.push_back(j);
+      in0.push_back(p.in0);
+      len.push_back(p.len);
+      row0.push_back(p.row0);
+      c0.push_back(nch);
+      nch += (p.len + CH - 1) / CH;
     }
   }
-  tc0[(size_t)nt] = (int32_t)ci0.size();
-  // per-chunk tables (small host-built plans, not per-pair data)
-  upload(g, S.chunk_i0, ci0.data(), ci0.size() * 8);
-  upload(g, S.in_base, cin.data(), cin.size() * 8);
-  upload(g, S.chunk_len, clen.data(), clen.size() * 4);
-  upload(g, S.chunk_trial, ctr.data(), ctr.size() * 4);
+  tc0[(size_t)nt] = (int32_t)nch;
+  c0.push_back(nch);
+  upload(g, S.p_trial, tr.data(), tr.size() * 4);
+  upload(g, S.p_in0, in0.data(), in0.size() * 8);
+  upload(g, S.p_len, len.data(), len.size() * 8);
+  upload(g, S.p_row0, row0.data(), row0.size() * 8);
+  upload(g, S.p_chunk0, c0.data(), c0.size() * 8);
   upload(g, S.trial_chunk0, tc0.data(), tc0.size() * 4);
-  return (int64_t)ci0.size();
+  need(g, S.chunk_i0, (size_t)nch * 8);
+  need(g, S.chunk_in0, (size_t)nch * 8);
+  need(g, S.chunk_len, (size_t)nch * 4);
+  need(g, S.chunk_trial, (size_t)nch * 4);
+  plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
+  plan.chunk_in0 = ptr<int64_t>(S.chunk_in0);
+  plan.chunk_len = ptr<int32_t>(S.chunk_len);
+  plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
+  plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
+  plan.nchunks = nch;
+  CK(group_chunk_tables(plan, ptr<int32_t>(S.p_trial), ptr<int64_t>(S.p_in0), ptr<int64_t>(S.p_len),
+                        ptr<int64_t>(S.p_row0), ptr<int64_t>(S.p_chunk0), (int32_t)tr.size(),
+                        g->stream));
+  return nch;
 }
 
 // Group `nt` trials whose pairs are given as pieces into out.members /
@@ -399,7 +419,8 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   const bool two = bits != bits1;
   const int64_t nbins = (int64_t)1 << bits;
   const int64_t nb1 = (int64_t)1 << bits1;
-  const int64_t nch = build_chunks(g, pieces, nt, S);
+  GroupArgs a;
+  const int64_t nch = build_pieces(g, pieces, nt, S, a.plan);
   std::vector<int64_t> seg((size_t)nt + 1);
   for (int j = 0; j <= nt; ++j) seg[(size_t)j] = seg_all[(size_t)t0 + j];
   upload(g, S.seg, seg.data(), seg.size() * 8);
@@ -418,20 +439,13 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   need(S.big_list, (size_t)(nt * nbins) * 8);             // big + mid lists
   need(S.big_count, 8);                                    // big + mid counts
   CK(cudaMemsetAsync(S.big_count.p, 0, 8, g->stream));
-  GroupArgs a;
   a.plan.c = nt;
   a.plan.bits = bits;
   a.plan.bits1 = bits1;
   a.plan.nbins = nbins;
   a.plan.nb1 = nb1;
-  a.plan.nchunks = nch;
   a.plan.npairs = npairs;
-  a.plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
-  a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
-  a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
-  a.plan.chunk_in0 = ptr<int64_t>(S.in_base);
   a.plan.seg = ptr<int64_t>(S.seg);
-  a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
   a.keys = keys;
   a.vals = vals;
   a.rowid = rowid;
@@ -565,20 +579,14 @@ void owner_partition(sg_graph *g, PassOut &P, KeyChunk &ch, GroupScratch &S,
       if (Bk[(size_t)b + 1] > Bk[(size_t)b])
         pieces.push_back(Piece{tl * nblk + b, (int64_t)tl * P.key_stride + Bk[(size_t)b],
                                Bk[(size_t)b + 1] - Bk[(size_t)b], Bk[(size_t)b]});
-  const int64_t nch = build_chunks(g, pieces, nvt, S);
+  GroupArgs a;
+  const int64_t nch = build_pieces(g, pieces, nvt, S, a.plan);
   need(g, S.counts, (size_t)(nch * R) * 4);
   need(g, S.bsize1, (size_t)nvt * R * 4);
   need(g, S.bstart1, (size_t)nvt * R * 4);
-  GroupArgs a;
   a.plan.c = nvt;
   a.plan.nb1 = R;
   a.plan.nbins = R;
-  a.plan.nchunks = nch;
-  a.plan.chunk_i0 = ptr<int64_t>(S.chunk_i0);
-  a.plan.chunk_len = ptr<int32_t>(S.chunk_len);
-  a.plan.chunk_trial = ptr<int32_t>(S.chunk_trial);
-  a.plan.chunk_in0 = ptr<int64_t>(S.in_base);
-  a.plan.trial_chunk0 = ptr<int32_t>(S.trial_chunk0);
   a.keys = ptr<uint64_t>(ch.keys);
   a.vals = nullptr;
   a.rowid = ptr<uint32_t>(P.rowid);

@@ -63,7 +63,7 @@ struct GroupPlan {
   int64_t nb1 = 1;           // 2^bits1
   int64_t nchunks = 0;
   int64_t npairs = 0;
-  // device tables
+  // device tables (built on the device from the piece table)
   int64_t *chunk_i0 = nullptr;     // [nchunks] row index of the chunk's first pair (implicit values)
   int32_t *chunk_len = nullptr;    // [nchunks]
   int32_t *chunk_trial = nullptr;  // [nchunks]
@@ -111,6 +111,11 @@ int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
 // Bucket plan for trial segments of at most `maxseg` pairs.
 void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
+// Fill plan.chunk_* (plan.nchunks entries) from the piece table (device
+// pointers; pieces ordered by trial, chunks of group_chunk_pairs() pairs).
+cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, const int64_t *p_in0,
+                               const int64_t *p_len, const int64_t *p_row0,
+                               const int64_t *p_chunk0, int32_t npieces, cudaStream_t st);
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
 cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
 cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st);   // chunk prefixes + bsize1 only

@@ -193,10 +193,20 @@ __global__ void __launch_bounds__(1024) colscan_kernel(const __grid_constant__ G
   const int64_t b = (int64_t)blockIdx.x * 32 + bl;
   const int k0 = g.plan.trial_chunk0[j], k1 = g.plan.trial_chunk0[j + 1];
   const int L = (k1 - k0 + 31) / 32;
-  const int a0 = k0 + pi * L, a1 = min(k1, a0 + L);
+  const int a0 = min(k1, k0 + pi * L), a1 = min(k1, a0 + L);
+  constexpr int U = 8;                     // loads in flight per thread
   uint32_t s = 0;
-  if (b < nb)
-    for (int k = a0; k < a1; ++k) s += g.counts[(int64_t)k * nb + b];
+  if (b < nb) {
+    int k = a0;
+    for (; k + U <= a1; k += U) {
+      uint32_t v[U];
+#pragma unroll
+      for (int x = 0; x < U; ++x) v[x] = g.counts[(int64_t)(k + x) * nb + b];
+#pragma unroll
+      for (int x = 0; x < U; ++x) s += v[x];
+    }
+    for (; k < a1; ++k) s += g.counts[(int64_t)k * nb + b];
+  }
   part[pi][bl] = s;
   __syncthreads();
   if (pi == 0) {
@@ -211,7 +221,18 @@ __global__ void __launch_bounds__(1024) colscan_kernel(const __grid_constant__ G
   __syncthreads();
   if (b < nb) {
     uint32_t run = part[pi][bl];
-    for (int k = a0; k < a1; ++k) {
+    int k = a0;
+    for (; k + U <= a1; k += U) {
+      uint32_t v[U];
+#pragma unroll
+      for (int x = 0; x < U; ++x) v[x] = g.counts[(int64_t)(k + x) * nb + b];
+#pragma unroll
+      for (int x = 0; x < U; ++x) {
+        g.counts[(int64_t)(k + x) * nb + b] = run;
+        run += v[x];
+      }
+    }
+    for (; k < a1; ++k) {
       uint32_t *p = g.counts + (int64_t)k * nb + b;
       const uint32_t v = *p;
       *p = run;
@@ -339,6 +360,30 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   }
 }
 
+// Per-chunk tables from the piece table (one thread per chunk; piece found
+// by binary search over the pieces' first chunks).
+__global__ void chunk_table_kernel(const int32_t *__restrict__ p_trial,
+                                   const int64_t *__restrict__ p_in0,
+                                   const int64_t *__restrict__ p_len,
+                                   const int64_t *__restrict__ p_row0,
+                                   const int64_t *__restrict__ p_chunk0, int32_t npieces,
+                                   int64_t nchunks, GroupPlan plan) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    int lo = 0, hi = npieces;        // p_chunk0[lo] <= k < p_chunk0[hi]
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (p_chunk0[mid] <= k) lo = mid;
+      else hi = mid;
+    }
+    const int64_t a = (k - p_chunk0[lo]) * kChunk;
+    plan.chunk_i0[k] = p_row0[lo] + a;
+    plan.chunk_in0[k] = p_in0[lo] + a;
+    plan.chunk_len[k] = (int32_t)min((int64_t)kChunk, p_len[lo] - a);
+    plan.chunk_trial[k] = p_trial[lo];
+  }
+}
+
 __global__ void popcount_kernel(const uint32_t *__restrict__ w, int64_t n, unsigned long long *out) {
   unsigned long long acc = 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
@@ -373,6 +418,17 @@ void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1) {
   while ((maxseg >> b) > target && b < kMaxBits) ++b;
   *bits = b;
   *bits1 = std::min(b, kCoarseBits);
+}
+
+cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, const int64_t *p_in0,
+                               const int64_t *p_len, const int64_t *p_row0,
+                               const int64_t *p_chunk0, int32_t npieces, cudaStream_t st) {
+  if (plan.nchunks == 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((plan.nchunks + 255) / 256, 148 * 8);
+  chunk_table_kernel<<<grid, 256, 0, st>>>(p_trial, p_in0, p_len, p_row0, p_chunk0, npieces,
+                                           plan.nchunks, plan);
+  ++g_launches;
+  return cudaGetLastError();
 }
 
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st) {
