@@ -114,57 +114,82 @@ __device__ __forceinline__ void warp_scan_1024(uint16_t *cnt) {
 
 // Stable placement pass: position of element e (visited in the order src,
 // identity if FIRST) = cursor[digit] + rank among same-digit peers of its
-// batch (__match_any_sync); the lowest peer advances the cursor.
+// batch (__match_any_sync, converged with the full mask; invalid lanes carry
+// the sentinel digit kWDigits); the lowest peer advances the packed-u16
+// cursor with a returning shared atomic, four batches in flight.
 template <bool FIRST>
 __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint16_t *src,
                                            uint16_t *cur, uint16_t *dst, int shift) {
   const int lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
-  for (int i0 = 0; i0 < n; i0 += 32) {
-    const int i = i0 + lane;
-    const bool valid = i < n;
-    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
-    if (valid) {
-      const uint16_t e = FIRST ? (uint16_t)i : src[i];
-      const uint32_t d = (S.d20[e] >> shift) & (kWDigits - 1);
-      const uint32_t m = __match_any_sync(vm, d);
-      const uint32_t rank = __popc(m & lt);
-      const uint32_t base = cur[d];
-      __syncwarp(vm);
-      if (rank == 0) cur[d] = (uint16_t)(base + __popc(m));
-      __syncwarp(vm);
-      dst[base + rank] = e;
+  uint32_t *cw = reinterpret_cast<uint32_t *>(cur);
+  for (int i0 = 0; i0 < n; i0 += 128) {
+    uint32_t e[4], d[4], m[4], o[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int i = i0 + u * 32 + lane;
+      const bool valid = i < n;
+      e[u] = valid ? (FIRST ? (uint32_t)i : (uint32_t)src[i]) : 0u;
+      d[u] = valid ? (S.d20[e[u]] >> shift) & (kWDigits - 1) : (uint32_t)kWDigits;
+      m[u] = __match_any_sync(0xffffffffu, d[u]);
+      o[u] = 0;
+      if (valid && (m[u] & lt) == 0)
+        o[u] = atomicAdd(&cw[d[u] >> 1], (uint32_t)__popc(m[u]) << ((d[u] & 1) << 4));
     }
-    __syncwarp();
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t oo = __shfl_sync(0xffffffffu, o[u], __ffs(m[u]) - 1);
+      if (i0 + u * 32 + lane < n) {
+        const uint32_t base = (oo >> ((d[u] & 1) << 4)) & 0xFFFFu;
+        dst[base + __popc(m[u] & lt)] = (uint16_t)e[u];
+      }
+    }
   }
+  __syncwarp();
 }
 
 // Write members (and sorted keys) in the order pm; head bits into S.hb.
 // Returns true if some adjacent pair is out of key order (a 20-bit tie).
+// Gathers of four batches are issued before their stores.
 __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n,
-                                          const uint16_t *pm, const uint64_t *Kg,
-                                          const uint32_t *Vg, int64_t gbase) {
+                                          const uint16_t *pm, const uint64_t *__restrict__ Kg,
+                                          const uint32_t *__restrict__ Vg, int64_t gbase) {
   const int lane = threadIdx.x & 31;
   bool bad = false;
   uint64_t carry = 0;
-  for (int p0 = 0; p0 < n; p0 += 32) {
-    const int p = p0 + lane;
-    const bool valid = p < n;
-    const int e = valid ? pm[p] : 0;
-    const uint64_t ke = valid ? Kg[e] : ~0ull;
-    const uint32_t ve = valid ? Vg[e] : 0u;
-    uint64_t prev = __shfl_up_sync(0xffffffffu, ke, 1);
-    if (lane == 0) prev = carry;
-    carry = __shfl_sync(0xffffffffu, ke, 31);
-    bool head = false;
-    if (valid) {
-      g.members[gbase + p] = ve;
-      if (g.okeys) g.okeys[gbase + p] = ke;
-      head = (p == 0) || prev != ke;
-      bad |= (p > 0) && ke < prev;
+  for (int p0 = 0; p0 < n; p0 += 128) {
+    int e[4];
+    uint64_t ke[4];
+    uint32_t ve[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int p = p0 + u * 32 + lane;
+      e[u] = p < n ? pm[p] : 0;
     }
-    const uint32_t hw = __ballot_sync(0xffffffffu, head);
-    if (lane == 0) S.hb[p0 >> 5] = hw;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const bool valid = p0 + u * 32 + lane < n;
+      ke[u] = valid ? Kg[e[u]] : ~0ull;
+      ve[u] = valid ? Vg[e[u]] : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      if (p0 + u * 32 >= n) break;                    // warp-uniform
+      const int p = p0 + u * 32 + lane;
+      const bool valid = p < n;
+      uint64_t prev = __shfl_up_sync(0xffffffffu, ke[u], 1);
+      if (lane == 0) prev = carry;
+      carry = __shfl_sync(0xffffffffu, ke[u], 31);
+      bool head = false;
+      if (valid) {
+        g.members[gbase + p] = ve[u];
+        if (g.okeys) g.okeys[gbase + p] = ke[u];
+        head = (p == 0) || prev != ke[u];
+        bad |= (p > 0) && ke[u] < prev;
+      }
+      const uint32_t hw = __ballot_sync(0xffffffffu, head);
+      if (lane == 0) S.hb[(p0 >> 5) + u] = hw;
+    }
   }
   return __any_sync(0xffffffffu, bad);
 }
