@@ -102,21 +102,29 @@ __device__ __forceinline__ void scan_all(const uint32_t *nb, int len, uint32_t a
   }
 }
 
-// Short rows (the staged tile pads each row to a multiple of 4): branch-free,
-// padding slots masked to +infinity, no remainder loop.
+// Short rows (pass-II rows average ~5 entries): whole quads branch-free, then
+// the 0-3 remaining entries as one pair and one single (row length is
+// warp-uniform: every lane scans the same row for its own trial), so no
+// padding slot is ever hashed.
 template <int S>
 __device__ __forceinline__ void scan_short(const uint32_t *nb, int len, uint32_t a, uint32_t b,
                                            uint32_t (&m)[S]) {
   const uint4 *nb4 = reinterpret_cast<const uint4 *>(nb);
-  const int nq = (len + 3) >> 2;
-  for (int q = 0; q < nq; ++q) {
-    const uint4 v = nb4[q];
-    const int e = q << 2;
+  int q = 0;
+  for (; q + 4 <= len; q += 4) {
+    const uint4 v = nb4[q >> 2];
     insert_min<S>(m, m31_hash(a, b, v.x));
-    insert_min<S>(m, e + 1 < len ? m31_hash(a, b, v.y) : 0xFFFFFFFFu);
-    insert_min<S>(m, e + 2 < len ? m31_hash(a, b, v.z) : 0xFFFFFFFFu);
-    insert_min<S>(m, e + 3 < len ? m31_hash(a, b, v.w) : 0xFFFFFFFFu);
+    insert_min<S>(m, m31_hash(a, b, v.y));
+    insert_min<S>(m, m31_hash(a, b, v.z));
+    insert_min<S>(m, m31_hash(a, b, v.w));
   }
+  if (len - q >= 2) {
+    const uint2 v = reinterpret_cast<const uint2 *>(nb)[q >> 1];
+    insert_min<S>(m, m31_hash(a, b, v.x));
+    insert_min<S>(m, m31_hash(a, b, v.y));
+    q += 2;
+  }
+  if (q < len) insert_min<S>(m, m31_hash(a, b, nb[q]));
 }
 
 template <int S>
