@@ -173,6 +173,8 @@ def roofline_table(stage_ms: dict, counts: dict, work: dict, pk: dict):
         # local: read 12 B pair + write 4 B member + 1 head bit per pair
         rows[f"hist{lv}"] = hbm_row(f"hist{lv}", 8 * P)
         rows[f"scatter{lv}"] = hbm_row(f"scatter{lv}", 20 * P)
+        # fine split (two-level plans): read 12 B pair + write 12 B pair
+        rows[f"fine{lv}"] = hbm_row(f"fine{lv}", 24 * P)
         rows[f"local{lv}"] = hbm_row(f"local{lv}", 16.125 * P)
     return {k: v for k, v in rows.items() if v}
 

@@ -175,7 +175,9 @@ SG_API sg_status sg_get_hash_params(sg_graph *g, int32_t level, uint32_t *A, uin
 
 /* Device milliseconds of the last stages (CUDA events on the handle's      */
 /* stream): [0] pass I, [1] group I, [2] pass II, [3] group II, then         */
-/* sub-stage detail.  *n receives the number written.     */
+/* sub-stages [4..17]: select1, hash1, select2, hash2, hist1, scatter1,      */
+/* local1, hist2, scatter2, local2, exchange1, exchange2, fine1, fine2       */
+/* (DESIGN.md §6).  At most 18 values; *n receives the number written.      */
 SG_API sg_status sg_get_stage_ms(const sg_graph *g, float *ms, int32_t cap, int32_t *n);
 
 /* Multi-GPU in-process test backend: `world` virtual ranks on one device,   */

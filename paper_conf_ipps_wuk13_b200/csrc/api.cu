@@ -306,6 +306,7 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
   a.keys = ptr<uint64_t>(ch.keys);
   a.key_stride = P.key_stride;
   a.counter = ptr<unsigned long long>(ctr);
+  a.tile_rows = st_hash == kStHash2 ? 16 : 8;   // pass II rows are short
   CK(minhash(a, g->num_sms, g->stream));
   dfree(g, ctr);
   st_end(g, st_hash);
@@ -473,8 +474,12 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   st_begin(g, st_scatter);
   CK(group_scatter(a, g->num_sms, g->stream));
   if (free_after_scatter) dfree(g, *free_after_scatter);   // keys consumed
-  if (two) CK(group_scatter2(a, g->stream));
   st_end(g, st_scatter);
+  if (two) {
+    st_begin(g, st_scatter == kStScatter1 ? kStFine1 : kStFine2);
+    CK(group_scatter2(a, g->stream));
+    st_end(g, st_scatter == kStScatter1 ? kStFine1 : kStFine2);
+  }
   st_begin(g, st_local);
   CK(group_local(a, g->num_sms, g->stream));
   st_end(g, st_local);

@@ -43,8 +43,9 @@ struct MinhashArgs {
   uint64_t *keys;                 // [nt][key_stride], key_stride % 8 == 0
   int64_t key_stride;
   unsigned long long *counter;    // zeroed device counter
+  int32_t tile_rows = 8;          // rows per warp tile: 8 (long rows) or 16 (short rows)
 };
-constexpr int kRowTile = 8;       // rows per warp tile (one 64 B store per trial)
+constexpr int kRowTile = 16;      // key_stride granule (multiple of every tile size)
 inline int64_t key_stride_for(int64_t nrows) { return (nrows + kRowTile - 1) / kRowTile * kRowTile; }
 cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st);
 

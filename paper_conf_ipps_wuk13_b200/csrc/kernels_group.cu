@@ -46,6 +46,17 @@ __device__ __forceinline__ uint32_t coarse_bin(uint64_t key, int64_t nb) {
   return (uint32_t)__umul64hi(key, (uint64_t)nb);
 }
 
+// The same bin when nb = 2^(64 - sh) is a power of two (sh = 64: one bin).
+__device__ __forceinline__ uint32_t coarse_bin_pow2(uint64_t key, int sh) {
+  return sh < 64 ? (uint32_t)(key >> sh) : 0u;
+}
+
+__device__ __forceinline__ int pow2_shift(int64_t nb) {
+  int l = 0;
+  while ((int64_t(1) << l) < nb) ++l;
+  return (int64_t(1) << l) == nb ? 64 - l : -1;   // -1: not a power of two
+}
+
 __device__ __forceinline__ uint32_t val_at(const GroupArgs &g, int64_t in_idx, int64_t i) {
   if (g.vals) return g.vals[in_idx];
   if (g.rowid) return g.rowid[i];
@@ -279,7 +290,8 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
   const int nb = (int)g.plan.nb1;
-  auto bin = [&](uint64_t key) { return coarse_bin(key, nb); };
+  const int sh = pow2_shift(nb);
+  auto bin = [&](uint64_t key) { return sh >= 0 ? coarse_bin_pow2(key, sh) : coarse_bin(key, nb); };
   uint64_t kk[kPerLane];
   uint32_t vv[kPerLane];
   int64_t k = blockIdx.x;

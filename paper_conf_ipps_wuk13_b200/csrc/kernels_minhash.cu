@@ -27,9 +27,11 @@ namespace {
 
 constexpr int kMhThreads = 256;
 constexpr int kMhWarps = kMhThreads / 32;
-constexpr int kNbCap = 1024;        // staged entries per warp (4 KB)
+// staged entries per warp: 4 KB for 8-row tiles of long rows, 2 KB for
+// 16-row tiles of short rows (the 16-row key buffer takes the difference)
+template <int TR>
+__host__ __device__ constexpr int nb_cap() { return TR == 8 ? 1024 : 512; }
 constexpr int kMaxPasses = 48;
-constexpr int TR = kRowTile;
 
 struct TrialPass {
   int16_t t0;      // first trial of the pass (relative to the launch's t0)
@@ -127,6 +129,38 @@ __device__ __forceinline__ void scan_short(const uint32_t *nb, int len, uint32_t
   if (q < len) insert_min<S>(m, m31_hash(a, b, nb[q]));
 }
 
+constexpr uint32_t kPad = 0xFFFFFFFFu;   // staged padding (vertex ids are < P < 2^31)
+
+// h of a staged word; padding words hash to all-ones (never among the minima)
+__device__ __forceinline__ uint32_t hash_or_pad(uint32_t A, uint32_t B, uint32_t v) {
+  return m31_hash(A, B, v) | (uint32_t)((int32_t)v >> 31);
+}
+
+// Two rows of QA / QB padded quads, scanned side by side (independent chains).
+template <int S, int QA, int QB>
+__device__ __forceinline__ void quads2(const uint32_t *pa, const uint32_t *pb, uint32_t A,
+                                       uint32_t B, uint32_t (&ma)[S], uint32_t (&mb)[S]) {
+  const uint4 *a4 = reinterpret_cast<const uint4 *>(pa);
+  const uint4 *b4 = reinterpret_cast<const uint4 *>(pb);
+#pragma unroll
+  for (int q = 0; q < (QA > QB ? QA : QB); ++q) {
+    if (q < QA) {
+      const uint4 v = a4[q];
+      insert_min<S>(ma, hash_or_pad(A, B, v.x));
+      insert_min<S>(ma, hash_or_pad(A, B, v.y));
+      insert_min<S>(ma, hash_or_pad(A, B, v.z));
+      insert_min<S>(ma, hash_or_pad(A, B, v.w));
+    }
+    if (q < QB) {
+      const uint4 v = b4[q];
+      insert_min<S>(mb, hash_or_pad(A, B, v.x));
+      insert_min<S>(mb, hash_or_pad(A, B, v.y));
+      insert_min<S>(mb, hash_or_pad(A, B, v.z));
+      insert_min<S>(mb, hash_or_pad(A, B, v.w));
+    }
+  }
+}
+
 template <int S>
 __device__ __forceinline__ void scan_any(const uint32_t *nb, int len, int part, int p, uint32_t a,
                                          uint32_t b, uint32_t (&m)[S]) {
@@ -134,12 +168,17 @@ __device__ __forceinline__ void scan_any(const uint32_t *nb, int len, int part, 
   else scan_strided<S>(nb, len, part, p, a, b, m);
 }
 
-template <int S>
-__global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_constant__ MhParams P) {
+// Per-warp key buffer slot of (row rr, trial lane tt): rows in 32-slot lines,
+// lanes XOR-swizzled by the row pair so that the coalesced store's reads of
+// one trial's rows fall in distinct banks.
+__device__ __forceinline__ int out_slot(int rr, int tt) { return rr * 32 + (tt ^ (rr >> 1)); }
+
+template <int S, int TR>
+__global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __grid_constant__ MhParams P) {
   extern __shared__ __align__(16) unsigned char smraw[];
   __shared__ int64_t sSt[kMhWarps][TR];
-  __shared__ int sLen[kMhWarps][TR];
-  __shared__ int sOff[kMhWarps][TR + 1];
+  __shared__ __align__(16) int sLen[kMhWarps][TR + 4];   // [TR]: read-ahead pad
+  __shared__ __align__(16) int sOff[kMhWarps][TR + 8];   // 16 B aligned rows
   const MinhashArgs &a = P.a;
   const int nt = a.nt;
   const int ntp = (nt + 7) & ~7;
@@ -149,7 +188,7 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
   uint32_t *sNbAll = reinterpret_cast<uint32_t *>(sOutAll + kMhWarps * TR * 32);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   uint64_t *sOut = sOutAll + w * TR * 32;
-  uint32_t *nb = sNbAll + w * kNbCap;
+  uint32_t *nb = sNbAll + w * nb_cap<TR>();
   for (int i = threadIdx.x; i < nt; i += blockDim.x) {
     sA[i] = a.A[a.t0 + i];
     sB[i] = a.B[a.t0 + i];
@@ -183,13 +222,13 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
       if (lane == 0) sOff[w][0] = 0;
       __syncwarp();
       const int total = sOff[w][TR];
-      if (total > kNbCap) {
+      if (total > nb_cap<TR>()) {
         // long rows: one row at a time, staged once (or chunk by chunk when it
         // exceeds the stage), all trial passes on it, scalar key stores
         for (int rr = 0; rr < nr; ++rr) {
           const int rl = sLen[w][rr];
           const uint32_t *src = a.entries + sSt[w][rr];
-          const bool fits = rl <= kNbCap;
+          const bool fits = rl <= nb_cap<TR>();
           if (fits) {
             __syncwarp();
             for (int i = lane; i < rl; i += 32) nb[i] = src[i];
@@ -209,8 +248,8 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
             if (fits) {
               scan_any<S>(nb, rl, part, p, A, B, m);
             } else {
-              for (int c0 = 0; c0 < rl; c0 += kNbCap) {
-                const int cl = min(kNbCap, rl - c0);
+              for (int c0 = 0; c0 < rl; c0 += nb_cap<TR>()) {
+                const int cl = min(nb_cap<TR>(), rl - c0);
                 __syncwarp();
                 for (int i = lane; i < cl; i += 32) nb[i] = src[c0 + i];
                 __syncwarp();
@@ -236,7 +275,7 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
 #pragma unroll
         for (int x = 1; x < TR; ++x) rr += (i >= sOff[w][x]);
         const int k = i - sOff[w][rr];
-        nb[i] = k < sLen[w][rr] ? a.entries[sSt[w][rr] + k] : 0u;
+        nb[i] = k < sLen[w][rr] ? a.entries[sSt[w][rr] + k] : kPad;   // pad: all-ones
       }
       __syncwarp();
       for (int pi = 0; pi < P.npass; ++pi) {
@@ -247,13 +286,49 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
         const int part = lane >> tp.logT;
         const int j = tp.t0 + tl;               // trial index within the launch
         const uint32_t A = sA[j], B = sB[j];
+        if (p == 1) {
+          // full 32-trial pass: rows of <= 8 entries go in pairs, straight-line
+          // over their padded quads (two independent chains per lane)
+          int rr = 0;
+          while (rr < nr) {
+            const int la = sLen[w][rr];
+            const int lb = rr + 1 < nr ? sLen[w][rr + 1] : 1 << 30;
+            if (la <= 8 && lb <= 8) {
+              const uint32_t *pa = nb + sOff[w][rr], *pb = nb + sOff[w][rr + 1];
+              uint32_t ma[S], mb[S];
+#pragma unroll
+              for (int i = 0; i < S; ++i) ma[i] = mb[i] = 0xFFFFFFFFu;
+              switch ((la > 4) * 2 + (lb > 4)) {
+                case 0: quads2<S, 1, 1>(pa, pb, A, B, ma, mb); break;
+                case 1: quads2<S, 1, 2>(pa, pb, A, B, ma, mb); break;
+                case 2: quads2<S, 2, 1>(pa, pb, A, B, ma, mb); break;
+                default: quads2<S, 2, 2>(pa, pb, A, B, ma, mb); break;
+              }
+              sOut[out_slot(rr, lane)] = fmix(shingle_id<S>(ma, a.seed, a.t0 + j));
+              sOut[out_slot(rr + 1, lane)] = fmix(shingle_id<S>(mb, a.seed, a.t0 + j));
+              rr += 2;
+            } else {
+              uint32_t m[S];
+#pragma unroll
+              for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+              if (la <= 24) scan_short<S>(nb + sOff[w][rr], la, A, B, m);
+              else scan_all<S>(nb + sOff[w][rr], la, A, B, m);
+              sOut[out_slot(rr, lane)] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+              rr += 1;
+            }
+          }
+        } else {
+        int rl_n = sLen[w][0], ro_n = sOff[w][0];   // row rr's metadata, loaded a row ahead
         for (int rr = 0; rr < nr; ++rr) {
-          const int rl = sLen[w][rr];
+          const int rl = rl_n;
+          const uint32_t *rnb = nb + ro_n;
+          rl_n = sLen[w][rr + 1];
+          ro_n = sOff[w][rr + 1];
           uint32_t m[S];
 #pragma unroll
           for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
-          if (p == 1 && rl <= 24) scan_short<S>(nb + sOff[w][rr], rl, A, B, m);
-          else scan_any<S>(nb + sOff[w][rr], rl, part, p, A, B, m);
+          if (p == 1 && rl <= 24) scan_short<S>(rnb, rl, A, B, m);
+          else scan_any<S>(rnb, rl, part, p, A, B, m);
           // merge the p partial lists of a trial (lanes tl, tl + T, ...)
           for (int o = T; o < 32; o <<= 1) {
             uint32_t x[S];
@@ -262,19 +337,27 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
 #pragma unroll
             for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
           }
-          if (part == 0) sOut[rr * 32 + tl] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+          if (part == 0) sOut[out_slot(rr, tl)] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+        }
         }
         __syncwarp();
-        if (part == 0) {
-          uint64_t *dst = a.keys + (int64_t)j * a.key_stride + r0;
-          if (nr == TR) {
-            ulonglong2 *d2 = reinterpret_cast<ulonglong2 *>(dst);
+        // coalesced stores: a trial's TR keys are TR * 8 contiguous bytes of
+        // its segment; consecutive lanes take consecutive 16 B pieces
+        if (nr == TR) {
+          constexpr int CPT = TR / 2;            // 16 B pieces per trial
 #pragma unroll
-            for (int q = 0; q < TR / 2; ++q)
-              d2[q] = make_ulonglong2(sOut[(2 * q) * 32 + tl], sOut[(2 * q + 1) * 32 + tl]);
-          } else {
-            for (int rr = 0; rr < nr; ++rr) dst[rr] = sOut[rr * 32 + tl];
+          for (int q = 0; q < CPT; ++q) {
+            const int c = q * 32 + lane;
+            const int tt = c / CPT, pp = c % CPT;
+            if (tt < T) {
+              const uint64_t k0 = sOut[out_slot(2 * pp, tt)], k1 = sOut[out_slot(2 * pp + 1, tt)];
+              *reinterpret_cast<ulonglong2 *>(a.keys + (int64_t)(tp.t0 + tt) * a.key_stride + r0 +
+                                              2 * pp) = make_ulonglong2(k0, k1);
+            }
           }
+        } else if (part == 0) {
+          uint64_t *dst = a.keys + (int64_t)j * a.key_stride + r0;
+          for (int rr = 0; rr < nr; ++rr) dst[rr] = sOut[out_slot(rr, tl)];
         }
         __syncwarp();
       }
@@ -282,12 +365,12 @@ __global__ void __launch_bounds__(kMhThreads) minhash_tile_kernel(const __grid_c
   }
 }
 
-template <int S>
-cudaError_t launch_tile(const MhParams &P, int num_sms, cudaStream_t st) {
+template <int S, int TR>
+cudaError_t launch_tile(MhParams &P, int num_sms, cudaStream_t st) {
   const int ntp = (P.a.nt + 7) & ~7;
   const size_t smem = (size_t)2 * ntp * 4 + (size_t)kMhWarps * TR * 32 * 8 +
-                      (size_t)kMhWarps * kNbCap * 4;
-  auto kern = minhash_tile_kernel<S>;
+                      (size_t)kMhWarps * nb_cap<TR>() * 4;
+  auto kern = minhash_tile_kernel<S, TR>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -295,11 +378,21 @@ cudaError_t launch_tile(const MhParams &P, int num_sms, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   per_sm = std::max(per_sm, 1);
   const int64_t ntiles = (P.a.nrows + TR - 1) / TR;
+  const int64_t warps = (int64_t)num_sms * 32;
+  P.tiles_per_grab = (int32_t)std::max<int64_t>(1, std::min<int64_t>(16, ntiles / (warps * 8)));
   const int64_t want = (ntiles + kMhWarps - 1) / kMhWarps;
   const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, std::max<int64_t>(want, 1));
   kern<<<grid, kMhThreads, smem, st>>>(P);
   ++g_launches;
   return cudaGetLastError();
+}
+
+// Short rows (pass II) take 16-row tiles: a trial's keys of one tile are a
+// full 128 B line; long rows (pass I) keep 8-row tiles (the stage holds them).
+template <int S>
+cudaError_t launch_s(MhParams &P, int num_sms, cudaStream_t st) {
+  if (P.a.tile_rows == 16) return launch_tile<S, 16>(P, num_sms, st);
+  return launch_tile<S, 8>(P, num_sms, st);
 }
 
 // ---- id recomputation for getters / report (one thread per request) --------
@@ -343,7 +436,8 @@ __global__ void shingle_ids_kernel(const int64_t *rstart, const int32_t *rlen,
 
 cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st) {
   if (a.nrows == 0 || a.nt == 0) return cudaSuccess;
-  if (a.key_stride % TR != 0) return cudaErrorInvalidValue;
+  if (a.key_stride % kRowTile != 0 || (a.tile_rows != 8 && a.tile_rows != 16))
+    return cudaErrorInvalidValue;
   MhParams P;
   P.a = a;
   // trial passes: full groups of 32 lanes (one trial per lane), then the
@@ -360,18 +454,15 @@ cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st) {
     }
   }
   P.npass = np;
-  const int64_t ntiles = (a.nrows + TR - 1) / TR;
-  const int64_t warps = (int64_t)num_sms * 32;
-  P.tiles_per_grab = (int32_t)std::max<int64_t>(1, std::min<int64_t>(16, ntiles / (warps * 8)));
   switch (a.s) {
-    case 1: return launch_tile<1>(P, num_sms, st);
-    case 2: return launch_tile<2>(P, num_sms, st);
-    case 3: return launch_tile<3>(P, num_sms, st);
-    case 4: return launch_tile<4>(P, num_sms, st);
-    case 5: return launch_tile<5>(P, num_sms, st);
-    case 6: return launch_tile<6>(P, num_sms, st);
-    case 7: return launch_tile<7>(P, num_sms, st);
-    case 8: return launch_tile<8>(P, num_sms, st);
+    case 1: return launch_s<1>(P, num_sms, st);
+    case 2: return launch_s<2>(P, num_sms, st);
+    case 3: return launch_s<3>(P, num_sms, st);
+    case 4: return launch_s<4>(P, num_sms, st);
+    case 5: return launch_s<5>(P, num_sms, st);
+    case 6: return launch_s<6>(P, num_sms, st);
+    case 7: return launch_s<7>(P, num_sms, st);
+    case 8: return launch_s<8>(P, num_sms, st);
     default: return cudaErrorInvalidValue;
   }
 }
