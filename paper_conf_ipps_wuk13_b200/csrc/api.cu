@@ -276,7 +276,11 @@ void plan_pass(sg_graph *g, PassOut &P) {
   }
   ct = std::min<int64_t>(ct, c);
   const int64_t nch = (c + ct - 1) / ct;
-  const int64_t per = (c + nch - 1) / nch;
+  int64_t per = (c + nch - 1) / nch;
+  // whole 32-trial groups per chunk: the min-hash runs 32 trials per lane
+  // pass and a tail pass (c mod 32 trials) costs a full pass per row, so
+  // e.g. 200 = 64+64+64+8 (7 passes) rather than 67+67+66 (11 passes)
+  if (per < c && per >= 32) per = per / 32 * 32;
   P.chunks.clear();
   for (int64_t t = 0; t < c; t += per) {
     KeyChunk k;

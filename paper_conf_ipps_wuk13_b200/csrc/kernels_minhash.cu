@@ -317,6 +317,21 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
               rr += 1;
             }
           }
+        } else if (TR == 16) {
+          // tail pass over short rows: the p lane groups take different rows
+          // (row rr = rb + part), each lane scanning a whole row for its trial
+          for (int rb = 0; rb < nr; rb += p) {
+            const int rr = rb + part;
+            if (rr < nr) {
+              const int rl = sLen[w][rr];
+              uint32_t m[S];
+#pragma unroll
+              for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+              if (rl <= 24) scan_short<S>(nb + sOff[w][rr], rl, A, B, m);
+              else scan_all<S>(nb + sOff[w][rr], rl, A, B, m);
+              sOut[out_slot(rr, tl)] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+            }
+          }
         } else {
         int rl_n = sLen[w][0], ro_n = sOff[w][0];   // row rr's metadata, loaded a row ahead
         for (int rr = 0; rr < nr; ++rr) {
