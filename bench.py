@@ -244,6 +244,13 @@ def bench_ours(args, rank, world, local_rank):
     et1 = float(deg[deg >= s1].sum()) * c1
     et2 = float(counts["entries2"]) * c2      # pass-II entries = sum |L| over S1'
     launches = counts["launches"]              # kernels of the last step (counter reset each step)
+    # Phase III on the device, outside the metric: clusters of
+    # >= 20 vertices (the size the paper evaluated)
+    phase3 = None
+    if world == 1:
+        _, ncl = B.report_dense_subgraphs(h, 0, 20, g.n)
+        phase3 = {"ms": round(B.sg_get_stage_ms(h).get("report", 0.0), 3), "clusters_ge20": int(ncl),
+                  "mode": "constituents (AMB-9)", "timed_in_metric": False}
     B.shingle_graph_destroy(h)
 
     # ---- e2e: the public API with host buffers, H2D + D2H inside the region
@@ -309,7 +316,7 @@ def bench_ours(args, rank, world, local_rank):
                    "l2": "inputs larger than L2 (CSR %.0f MB; per-step intermediates several GB)" % ((g.row_ptr.nbytes + g.col.nbytes) / 1e6),
                    "parallelism": f"vertex-range shards x{world}"},
         "stage_ms": {k: round(v, 3) for k, v in stage_ms.items() if v > 0},
-        "roofline": dom, "roofline_stages": rt, "peak_source": pk["src"],
+        "roofline": dom, "roofline_stages": rt, "peak_source": pk["src"], "phase3": phase3,
         "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches * args.steps,
         "gpu_launches_per_step": launches,
         "clocks": clocks,

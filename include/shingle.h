@@ -49,6 +49,7 @@ typedef struct sg_graph sg_graph;
 /* create() flags */
 #define SG_DEVICE_PTRS 0x1u   /* row_ptr / col are device pointers (on dist->device) */
 #define SG_NO_VALIDATE 0x2u   /* skip the CSR validation (caller guarantees it)   */
+#define SG_REPORT_HOST 0x10   /* report_dense_subgraphs mode flag: host union-find */
 
 /* Multi-GPU description: one process (or, with loopback, one host thread) per
  * rank, vertex-range sharding, owner-routed exchange before each grouping
@@ -121,7 +122,11 @@ SG_API sg_status group_by_shingle(sg_graph *g);
 /*              reported as singletons (labels[v] = v).                      */
 /*   n_clusters receives the number of clusters with >= max(2, min_size)     */
 /*              vertices (may be NULL).                                      */
-/* Host work, outside the timed hot path.  Requires state GROUPED2 and      */
+/*   mode       0 or 1, optionally | SG_REPORT_HOST.  Default: on the device */
+/*              (lock-free union-find over n, one thread per S1' node and per  */
+/*              G_II pair, stage "report" of sg_get_stage_ms); with the flag:  */
+/*              the same union-find on the host (G_I, G_II copied back).       */
+/* Outside the timed two-pass hot path.  Requires state GROUPED2 and         */
 /* world == 1 (SG_ESTATE otherwise: gather G_II with sg_get_groups).         */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
@@ -175,9 +180,9 @@ SG_API sg_status sg_get_hash_params(sg_graph *g, int32_t level, uint32_t *A, uin
 
 /* Device milliseconds of the last stages (CUDA events on the handle's      */
 /* stream): [0] pass I, [1] group I, [2] pass II, [3] group II, then         */
-/* sub-stages [4..17]: select1, hash1, select2, hash2, hist1, scatter1,      */
-/* local1, hist2, scatter2, local2, exchange1, exchange2, fine1, fine2       */
-/* (DESIGN.md §6).  At most 18 values; *n receives the number written.      */
+/* sub-stages [4..18]: select1, hash1, select2, hash2, hist1, scatter1,      */
+/* local1, hist2, scatter2, local2, exchange1, exchange2, fine1, fine2,      */
+/* report.  At most 19 values; *n receives the number written.*/
 SG_API sg_status sg_get_stage_ms(const sg_graph *g, float *ms, int32_t cap, int32_t *n);
 
 /* Multi-GPU in-process test backend: `world` virtual ranks on one device,   */

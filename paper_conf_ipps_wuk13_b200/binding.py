@@ -24,7 +24,8 @@ STATUS_NAMES = {0: "SG_OK", 1: "SG_EINVAL", 2: "SG_ENOMEM", 3: "SG_ESTATE", 4: "
                 5: "SG_ENCCL", 6: "SG_EOVERFLOW"}
 STAGES = ["pass1", "group1", "pass2", "group2", "select1", "hash1", "select2", "hash2",
           "hist1", "scatter1", "local1", "hist2", "scatter2", "local2", "exchange1", "exchange2",
-          "fine1", "fine2"]
+          "fine1", "fine2", "report"]
+SG_REPORT_HOST = 0x10
 
 
 class SGError(RuntimeError):

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -225,6 +226,20 @@ __global__ void rebase_kernel(int64_t *rp, int64_t n1, int64_t base) {
 // ---------------------------------------------------------------- HBM planning
 // Bytes the handle may still allocate: free device memory + blocks cached by
 // the stream-ordered pool, capped by the SG_MEM_BUDGET test hook.
+// SG_DEBUG_HOST: host-side timeline of the pass/group calls on stderr
+// (diagnostics for the host gaps inside the stage events).
+struct HostMark {
+  bool on = getenv("SG_DEBUG_HOST") != nullptr;
+  std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+  void operator()(const char *what) {
+    if (!on) return;
+    const auto t = std::chrono::steady_clock::now();
+    fprintf(stderr, "[sg-host] %-24s %8.3f ms\n", what,
+            std::chrono::duration<double, std::milli>(t - t0).count());
+    t0 = t;
+  }
+};
+
 int64_t avail_bytes(sg_graph *g) {
   size_t fr = 0, tot = 0;
   CK(cudaMemGetInfo(&fr, &tot));
@@ -960,6 +975,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     P.hB.resize((size_t)c);
     hash_pairs(seed, c, P.hA.data(), P.hB.data());
     const int st_all = level == 0 ? kStPass1 : kStPass2;
+    HostMark hm;
     st_begin(g, st_all);
     st_begin(g, level == 0 ? kStSelect1 : kStSelect2);
     dalloc(g, P.A, (size_t)c * 4);
@@ -977,6 +993,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
                           g->stream));
       CK(cudaMemcpyAsync(&nrows, tot.p, 8, cudaMemcpyDeviceToHost, g->stream));
       sync(g);
+      hm("select count + sync");
       dalloc(g, P.rstart, (size_t)nrows * 8);
       dalloc(g, P.rlen, (size_t)nrows * 4);
       dalloc(g, P.rowid, (size_t)nrows * 4);
@@ -1014,12 +1031,16 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     if (level == 1 && g->s1p_global >= (int64_t)0xFFFFFFFFll)
       fail(g, SG_EOVERFLOW, "|S1'| exceeds 2^32 - 1 (members are u32)");
     st_end(g, level == 0 ? kStSelect1 : kStSelect2);
+    hm("select write enqueued");
     // ---- min-hash top-s of every row and trial (the hot kernel)
     plan_pass(g, P);
+    hm("plan_pass");
     if (!P.deferred)
       for (auto &ch : P.chunks) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+    hm("min-hash enqueued");
     st_end(g, st_all);
     sync(g);
+    hm("pass done (sync)");
     g->state = level == 0 ? kPassed1 : kPassed2;
   }, true);
 }
@@ -1277,11 +1298,56 @@ sg_status sg_get_stage_ms(const sg_graph *gc, float *ms, int32_t cap, int32_t *n
 sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
                                  int64_t *n_clusters) {
   return guarded(g, [&] {
-    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
+    const bool host = (mode & SG_REPORT_HOST) != 0;
+    mode &= ~SG_REPORT_HOST;
+    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1 (| SG_REPORT_HOST)");
     if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
     if (g->world > 1) require_single(g, "report_dense_subgraphs");
     PassOut &P1 = g->pass[0];
     PassOut &P2 = g->pass[1];
+    if (!host) {
+      // ---- device union-find (kernels_report.cu)
+      ReportArgs a;
+      a.n = g->n;
+      a.mode = mode;
+      a.min_size = min_size;
+      a.s1 = P1.s;
+      a.s2 = P2.s;
+      a.A1 = ptr<uint32_t>(P1.A);
+      a.B1 = ptr<uint32_t>(P1.B);
+      a.A2 = ptr<uint32_t>(P2.A);
+      a.B2 = ptr<uint32_t>(P2.B);
+      a.row_ptr = ptr<int64_t>(g->row_ptr);
+      a.col = ptr<uint32_t>(g->col);
+      a.members1 = ptr<uint32_t>(g->grp[0].members);
+      a.rows1 = P1.nrows;
+      a.rstart2 = ptr<int64_t>(P2.rstart);
+      a.rlen2 = ptr<int32_t>(P2.rlen);
+      a.nk = P2.nrows;
+      a.members2 = ptr<uint32_t>(g->grp[1].members);
+      a.head2 = ptr<uint32_t>(g->grp[1].head);
+      a.npairs2 = g->grp[1].npairs;
+      a.rows2 = P2.nrows;
+      DBuf parent, rep1, size, dlab, dnc;
+      dalloc(g, parent, (size_t)a.n * 4);
+      dalloc(g, rep1, (size_t)a.nk * 4);
+      dalloc(g, size, (size_t)a.n * 4);
+      dalloc(g, dlab, (size_t)a.n * 4);
+      dalloc(g, dnc, 8);
+      g->st[kStReport].clear();
+      st_begin(g, kStReport);
+      CK(report_device(a, ptr<uint32_t>(parent), ptr<uint32_t>(rep1), ptr<uint32_t>(size),
+                       ptr<int32_t>(dlab), ptr<unsigned long long>(dnc), g->num_sms, g->stream));
+      st_end(g, kStReport);
+      unsigned long long nc = 0;
+      if (labels)
+        CK(cudaMemcpyAsync(labels, dlab.p, (size_t)a.n * 4, cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaMemcpyAsync(&nc, dnc.p, 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      for (DBuf *b : {&parent, &rep1, &size, &dlab, &dnc}) dfree(g, *b);
+      if (n_clusters) *n_clusters = (int64_t)nc;
+      return;
+    }
     HostGroups H1, H2;
     host_groups(g, 0, H1, true);
     host_groups(g, 1, H2, mode == 0);

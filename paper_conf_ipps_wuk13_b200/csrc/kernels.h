@@ -126,6 +126,30 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level 
 // mid and big tiers over the lists the warp tier filled (no host sync).
 cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
 
+// ---- Phase III on the device (kernels_report.cu) ---------------------------
+struct ReportArgs {
+  int64_t n = 0;                    // vertices of G
+  int32_t mode = 0;                 // 0 constituents, 1 generators (AMB-9)
+  int32_t min_size = 1;
+  int32_t s1 = 0, s2 = 0;
+  const uint32_t *A1 = nullptr, *B1 = nullptr, *A2 = nullptr, *B2 = nullptr;   // device [c]
+  const int64_t *row_ptr = nullptr; // CSR of G (device, single rank: rebased = global)
+  const uint32_t *col = nullptr;
+  const uint32_t *members1 = nullptr;   // G_I members (canonical order)
+  int64_t rows1 = 0;                // pass-I rows: trial j owns members1[j*rows1, (j+1)*rows1)
+  const int64_t *rstart2 = nullptr; // S1' node k: its group L(k) = members1[rstart2[k], +rlen2[k])
+  const int32_t *rlen2 = nullptr;
+  int64_t nk = 0;                   // |S1'|
+  const uint32_t *members2 = nullptr;   // G_II members (S1' indices)
+  const uint32_t *head2 = nullptr;      // G_II head bits
+  int64_t npairs2 = 0;
+  int64_t rows2 = 0;                // pass-II rows (= nk): trial t owns [t*rows2, (t+1)*rows2)
+};
+// parent/size: device uint32[n]; rep1: device uint32[nk]; labels: device
+// int32[n]; *d_nc receives the cluster count.
+cudaError_t report_device(const ReportArgs &a, uint32_t *parent, uint32_t *rep1, uint32_t *size,
+                          int32_t *labels, unsigned long long *d_nc, int num_sms, cudaStream_t st);
+
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);

@@ -110,14 +110,15 @@ struct Groups {
   DBuf okeys;                          // uint64 [npairs] sorted keys (multi-rank only)
 };
 
-constexpr int kNumStages = 18;
+constexpr int kNumStages = 19;
 enum StageId {
   kStPass1 = 0, kStGroup1 = 1, kStPass2 = 2, kStGroup2 = 3,
   kStSelect1 = 4, kStHash1 = 5, kStSelect2 = 6, kStHash2 = 7,
   kStHist1 = 8, kStScatter1 = 9, kStLocal1 = 10,
   kStHist2 = 11, kStScatter2 = 12, kStLocal2 = 13,
   kStX1 = 14, kStX2 = 15,
-  kStFine1 = 16, kStFine2 = 17     // second-level (fine) split of two-level plans
+  kStFine1 = 16, kStFine2 = 17,    // second-level (fine) split of two-level plans
+  kStReport = 18                   // Phase III on the device (outside the metric)
 };
 
 struct Exchange;  // multi-GPU (exchange.cu)

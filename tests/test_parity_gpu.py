@@ -29,8 +29,10 @@ def run_both(B, g, s1, c1, seed1, s2, c2, seed2, report=True):
             M2=B.sg_get_shingles(G.h, 2), G2=B.sg_get_groups(G.h, 2), counts=B.sg_get_counts(G.h),
             A1=B.sg_get_hash_params(G.h, 1, c1), A2=B.sg_get_hash_params(G.h, 2, c2))
         if report:
-            out["rep0"] = G.report(0)
+            out["rep0"] = G.report(0)                        # device union-find (default)
             out["rep1"] = G.report(1, 3)
+            out["rep0h"] = G.report(0 | B.SG_REPORT_HOST)    # host union-find
+            out["rep1h"] = G.report(1 | B.SG_REPORT_HOST, 3)
     ref = oracle.shingling(g.row_ptr, g.col, s1, c1, seed1, s2, c2, seed2)
     return out, ref
 
@@ -63,6 +65,9 @@ def assert_parity(out, ref, report=True):
         l1, n1 = out["rep1"]
         r1, m1 = ref.report(1, 3)
         assert n1 == m1 and np.array_equal(l1, r1)
+        for key, (rl, rn) in (("rep0h", (r0, m0)), ("rep1h", (r1, m1))):
+            lh, nh = out[key]
+            assert nh == rn and np.array_equal(lh, rl), key
 
 
 def test_tiny_config_full_parity(B):
