@@ -142,6 +142,11 @@ def cpu_model():
 
 
 # ---------------------------------------------------------------- roofline
+# ncu-measured DRAM traffic per pair of the level-II kernels on gos2m (c2 = 64
+# capture, profiles/round1_gos2m_v5_ncu_full.md): hist 21.36 GB, scatter
+# 69.80 GB, fine split 92.96 GB, warp-tier local sort 43.23 GB for 2.588e9 pairs
+NCU_BYTES_PER_PAIR = {"hist2": 8.25, "scatter2": 26.97, "fine2": 35.92, "local2": 16.70}
+
 def roofline_table(stage_ms: dict, counts: dict, work: dict, pk: dict):
     """Per-kernel algorithmic work / device time."""
     hbm = pk["hbm"]
@@ -296,7 +301,16 @@ def bench_ours(args, rank, world, local_rank):
     dom = dict(rt[dom_name]) if dom_name else None
     if dom:
         dom["kernel"] = dom_name
-        dom["traffic"] = None
+        # DRAM bytes (read + write) per pair of the dominant kernel, measured by
+        # `ncu --set full` on the same workload at c2 = 64 (one launch of each
+        # level-II kernel; profiles/round1_gos2m_v5_ncu_full.md), scaled to the
+        # pairs this stage processes per step
+        tr = NCU_BYTES_PER_PAIR.get(dom_name)
+        lv = dom_name[-1]
+        npairs = counts.get(f"pairs{lv}", 0)
+        dom["traffic"] = int(tr * npairs) if (tr and args.config == "gos2m") else None
+        dom["traffic_source"] = ("ncu dram__bytes_read.sum + dram__bytes_write.sum per pair "
+                                 "(profiles/round1_gos2m_v5_ncu_full.md) x pairs of the stage")
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         v, dt, u, nnz_s = run_oracle(g, cfg, args.cpu_sample_nnz)
