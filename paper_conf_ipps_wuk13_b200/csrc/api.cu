@@ -309,8 +309,8 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
   st_begin(g, st_hash);
   dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
   DBuf ctr;
-  dalloc(g, ctr, 8);
-  CK(cudaMemsetAsync(ctr.p, 0, 8, g->stream));
+  dalloc(g, ctr, 16);
+  CK(cudaMemsetAsync(ctr.p, 0, 16, g->stream));
   MinhashArgs a;
   a.rstart = ptr<int64_t>(P.rstart);
   a.rlen = ptr<int32_t>(P.rlen);
@@ -325,6 +325,7 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
   a.keys = ptr<uint64_t>(ch.keys);
   a.key_stride = P.key_stride;
   a.counter = ptr<unsigned long long>(ctr);
+  a.hub_counter = a.counter + 1;
   a.tile_rows = st_hash == kStHash2 ? 16 : 8;   // pass II rows are short
   CK(minhash(a, g->num_sms, g->stream));
   dfree(g, ctr);

@@ -42,7 +42,8 @@ struct MinhashArgs {
   uint64_t seed;
   uint64_t *keys;                 // [nt][key_stride], key_stride % 8 == 0
   int64_t key_stride;
-  unsigned long long *counter;    // zeroed device counter
+  unsigned long long *counter;    // zeroed device counter (row tiles)
+  unsigned long long *hub_counter;  // zeroed device counter (hub-row blocks)
   int32_t tile_rows = 8;          // rows per warp tile: 8 (long rows) or 16 (short rows)
 };
 constexpr int kRowTile = 16;      // key_stride granule (multiple of every tile size)

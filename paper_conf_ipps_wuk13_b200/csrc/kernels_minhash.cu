@@ -27,6 +27,10 @@ namespace {
 
 constexpr int kMhThreads = 256;
 constexpr int kMhWarps = kMhThreads / 32;
+// Rows longer than this (hub vertices) are left to the block-per-vertex
+// hub_kernel: one CTA per row, the row split over its 8 warps.
+constexpr int kHubLen = 2048;
+
 // staged entries per warp: 4 KB for 8-row tiles of long rows, 2 KB for
 // 16-row tiles of short rows (the 16-row key buffer takes the difference)
 template <int TR>
@@ -227,6 +231,7 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
         // exceeds the stage), all trial passes on it, scalar key stores
         for (int rr = 0; rr < nr; ++rr) {
           const int rl = sLen[w][rr];
+          if (rl > kHubLen) continue;                 // block-per-vertex kernel (hub_kernel)
           const uint32_t *src = a.entries + sSt[w][rr];
           const bool fits = rl <= nb_cap<TR>();
           if (fits) {
@@ -380,6 +385,108 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
   }
 }
 
+// Block-per-vertex min-hash of hub rows (len > kHubLen): the CTA scans its
+// share of the rows' lengths; each hub found is processed by the whole CTA.
+// The row is staged in shared memory (kHubStage entries at a time,
+// coalesced) and every trial pass reads it from there: warp w takes the w-th
+// eighth of the staged quads, lane = trial (full passes) or (trial,
+// neighbour part) (tail passes), 128-bit broadcast loads, four hashes per
+// load; the eight partial top-s lists of a trial are merged through shared
+// memory.  Rows longer than the stage are re-staged per pass.
+constexpr int kHubStage = 16384;                 // entries (64 KB)
+
+template <int S>
+__global__ void __launch_bounds__(kMhThreads) hub_kernel(const __grid_constant__ MhParams P) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  uint32_t *stg = reinterpret_cast<uint32_t *>(smraw);
+  __shared__ uint32_t sPart[kMhWarps][32][S];
+  __shared__ int sHub[kMhThreads];
+  __shared__ int sNHub;
+  const MinhashArgs &a = P.a;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  __shared__ int64_t sB0;
+  for (;;) {
+    // row blocks grabbed dynamically (hubs are few and unevenly spread)
+    if (threadIdx.x == 0) {
+      sNHub = 0;
+      sB0 = (int64_t)atomicAdd(a.hub_counter, 1ull) * kMhThreads;
+    }
+    __syncthreads();
+    const int64_t b0 = sB0;
+    if (b0 >= a.nrows) break;
+    const int64_t r = b0 + threadIdx.x;
+    if (r < a.nrows && a.rlen[r] > kHubLen) sHub[atomicAdd(&sNHub, 1)] = threadIdx.x;
+    __syncthreads();
+    const int nh = sNHub;
+    for (int hI = 0; hI < nh; ++hI) {
+      const int64_t row = b0 + sHub[hI];
+      const int len = a.rlen[row];
+      const uint32_t *src = a.entries + a.rstart[row];
+      const bool once = len <= kHubStage;
+      if (once) {
+        __syncthreads();
+        for (int i = threadIdx.x; i < len; i += kMhThreads) stg[i] = src[i];
+        __syncthreads();
+      }
+      for (int pi = 0; pi < P.npass; ++pi) {
+        const TrialPass tp = P.pass[pi];
+        const int T = 1 << tp.logT;
+        const int p = 1 << tp.logp;
+        const int tl = lane & (T - 1);
+        const int part = lane >> tp.logT;
+        const int j = tp.t0 + tl;
+        const uint32_t A = a.A[a.t0 + j], B = a.B[a.t0 + j];
+        uint32_t m[S];
+#pragma unroll
+        for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+        for (int c0 = 0; c0 < len; c0 += kHubStage) {
+          const int cl = min(kHubStage, len - c0);
+          if (!once) {
+            __syncthreads();
+            for (int i = threadIdx.x; i < cl; i += kMhThreads) stg[i] = src[c0 + i];
+            __syncthreads();
+          }
+          const int nq = cl >> 2;
+          const int q0 = nq * w / kMhWarps, q1 = nq * (w + 1) / kMhWarps;
+          const uint4 *s4 = reinterpret_cast<const uint4 *>(stg);
+#pragma unroll 2
+          for (int q = q0 + part; q < q1; q += p) {
+            const uint4 v = s4[q];
+            const uint32_t h0 = m31_hash(A, B, v.x), h1 = m31_hash(A, B, v.y);
+            const uint32_t h2 = m31_hash(A, B, v.z), h3 = m31_hash(A, B, v.w);
+            if (min(min(h0, h1), min(h2, h3)) < m[S - 1]) {
+              insert_min<S>(m, h0);
+              insert_min<S>(m, h1);
+              insert_min<S>(m, h2);
+              insert_min<S>(m, h3);
+            }
+          }
+          if (w == kMhWarps - 1)                        // the 0-3 entries after the last quad
+            for (int e = (nq << 2) + part; e < cl; e += p) insert_min<S>(m, m31_hash(A, B, stg[e]));
+        }
+        for (int o = T; o < 32; o <<= 1) {
+          uint32_t x[S];
+#pragma unroll
+          for (int i = 0; i < S; ++i) x[i] = __shfl_xor_sync(0xffffffffu, m[i], o);
+#pragma unroll
+          for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < S; ++i) sPart[w][lane][i] = m[i];
+        __syncthreads();
+        if (w == 0 && part == 0) {
+          for (int x = 1; x < kMhWarps; ++x)
+#pragma unroll
+            for (int i = 0; i < S; ++i) insert_min<S>(m, sPart[x][lane][i]);
+          a.keys[(int64_t)j * a.key_stride + row] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+        }
+        __syncthreads();
+      }
+    }
+    __syncthreads();
+  }
+}
+
 template <int S, int TR>
 cudaError_t launch_tile(MhParams &P, int num_sms, cudaStream_t st) {
   const int ntp = (P.a.nt + 7) & ~7;
@@ -398,6 +505,14 @@ cudaError_t launch_tile(MhParams &P, int num_sms, cudaStream_t st) {
   const int64_t want = (ntiles + kMhWarps - 1) / kMhWarps;
   const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, std::max<int64_t>(want, 1));
   kern<<<grid, kMhThreads, smem, st>>>(P);
+  ++g_launches;
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  // hub rows (block per vertex); the tile kernel skipped them
+  const size_t hsm = (size_t)kHubStage * 4;
+  if ((e = cudaFuncSetAttribute(hub_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)hsm)) != cudaSuccess)
+    return e;
+  hub_kernel<S><<<num_sms * 3, kMhThreads, hsm, st>>>(P);
   ++g_launches;
   return cudaGetLastError();
 }

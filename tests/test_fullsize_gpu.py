@@ -1,0 +1,105 @@
+"""Full-size parity on the bench workload (BASELINE configs[1], gos2m: 2M
+vertices, 56.9M edges, s1 = s2 = 2, c1 = c2 = 200), in the launch
+configuration bench.py times (one GPU, the same trial chunking).
+
+The oracle cannot run the whole method at this size in seconds, so the checks
+are (a) sampled outputs the oracle computes one by one (pass-I shingle rows)
+and (b) properties that hold at any size: the selected rows, the canonical
+order of G_I, each sampled group's members sharing its id, the S1' filter,
+and the pair / entry counts of both levels.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from synth import graphs as SG
+
+pytestmark = pytest.mark.gpu
+
+M1 = np.uint64(0xbf58476d1ce4e5b9)
+M2 = np.uint64(0x94d049bb133111eb)
+
+
+def mix64_np(z):
+    """splitmix64 finaliser on a uint64 array (the grouping key, AMB-19)."""
+    z = z.copy()
+    with np.errstate(over="ignore"):
+        z = (z ^ (z >> np.uint64(30))) * M1
+        z = (z ^ (z >> np.uint64(27))) * M2
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+@pytest.fixture(scope="module")
+def run():
+    import torch
+    torch.cuda.init()
+    from paper_conf_ipps_wuk13_b200 import binding as B
+    g = SG.make("gos2m")
+    cfg = SG.CONFIGS["gos2m"]
+    h = B.shingle_graph_create(g.row_ptr, g.col)
+    B.shingle_pass(h, cfg["s1"], cfg["c1"], cfg["seed1"])
+    B.group_by_shingle(h)
+    B.shingle_pass(h, cfg["s2"], cfg["c2"], cfg["seed2"])
+    B.group_by_shingle(h)
+    out = dict(counts=B.sg_get_counts(h), M1=B.sg_get_shingles(h, 1), G1=B.sg_get_groups(h, 1),
+               s1p=B.sg_get_s1p(h), A1=B.sg_get_hash_params(h, 1, cfg["c1"]))
+    B.shingle_graph_destroy(h)
+    return g, cfg, out
+
+
+def test_fullsize_rows_and_sampled_pass1_shingles(run):
+    g, cfg, out = run
+    ids1, rows1 = out["M1"]
+    deg = np.diff(g.row_ptr)
+    assert np.array_equal(rows1, np.flatnonzero(deg >= cfg["s1"]).astype(np.uint32))
+    A, B = out["A1"]
+    rng = np.random.default_rng(7)
+    for i in rng.choice(len(rows1), 600, replace=False):
+        u = int(rows1[i])
+        row = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
+        want = oracle.row_shingles(row, cfg["s1"], cfg["c1"], cfg["seed1"], A, B)
+        assert np.array_equal(ids1[i], want), f"pass-I shingles of vertex {u}"
+
+
+def test_fullsize_group1_canonical_and_sampled_members(run):
+    g, cfg, out = run
+    ids1, rows1 = out["M1"]
+    tg, gid, offs, mem = out["G1"]
+    c1 = cfg["c1"]
+    n_e = len(rows1)
+    assert tg[0] == 0 and tg[-1] == len(gid) and np.all(np.diff(tg) > 0)
+    assert offs[-1] == len(mem) == n_e * c1
+    sizes = np.diff(offs)
+    assert sizes.min() >= 1
+    # canonical order: per trial, keys mix64(id) strictly ascending
+    key = mix64_np(gid)
+    for j in range(c1):
+        k = key[tg[j]:tg[j + 1]]
+        assert np.all(k[1:] > k[:-1]), f"trial {j} keys not strictly ascending"
+        # each trial segment holds every generator exactly once
+        assert offs[tg[j + 1]] - offs[tg[j]] == n_e
+    rng = np.random.default_rng(11)
+    trial_of = np.searchsorted(tg, np.arange(len(gid)), side="right") - 1
+    for q in rng.choice(len(gid), 2000, replace=False):
+        L = mem[offs[q]:offs[q + 1]]
+        assert np.all(L[1:] > L[:-1]), "members strictly ascending"
+        pos = np.searchsorted(rows1, L)
+        assert np.array_equal(rows1[pos], L)
+        assert np.all(ids1[pos, trial_of[q]] == gid[q]), "members generate the group's shingle"
+
+
+def test_fullsize_s1p_filter_and_level2_counts(run):
+    g, cfg, out = run
+    ids1, rows1 = out["M1"]
+    tg, gid, offs, mem = out["G1"]
+    c = out["counts"]
+    sizes = np.diff(offs)
+    sel = np.flatnonzero(sizes >= cfg["s2"])
+    s1p, k0 = out["s1p"]
+    assert k0 == 0 and np.array_equal(s1p, sel)
+    assert c["n_e"] == len(rows1) and c["groups1"] == len(gid) and c["pairs1"] == len(mem)
+    assert c["s1p"] == len(sel)
+    assert c["entries2"] == int(sizes[sel].sum())
+    assert c["pairs2"] == len(sel) * cfg["c2"]
+    assert len(sel) <= c["groups2"] <= c["pairs2"]
