@@ -139,15 +139,15 @@ int ev_take(sg_graph *g) {
   return (int)g->ev_next++;
 }
 
-void st_begin(sg_graph *g, int id) {
+void st_begin(sg_graph *g, int id, cudaStream_t st = nullptr) {
   const int e = ev_take(g);
-  CK(cudaEventRecord(g->ev_pool[(size_t)e], g->stream));
+  CK(cudaEventRecord(g->ev_pool[(size_t)e], st ? st : g->stream));
   g->st[id].push_back({e, -1});
 }
 
-void st_end(sg_graph *g, int id) {
+void st_end(sg_graph *g, int id, cudaStream_t st = nullptr) {
   const int e = ev_take(g);
-  CK(cudaEventRecord(g->ev_pool[(size_t)e], g->stream));
+  CK(cudaEventRecord(g->ev_pool[(size_t)e], st ? st : g->stream));
   g->st[id].back().second = e;
 }
 
@@ -185,8 +185,15 @@ sg_status guarded(sg_graph *g, F &&f, bool collective = false) {
 }
 
 void free_pass(sg_graph *g, PassOut &p) {
+  bool side = false;
+  for (auto &ch : p.chunks) side |= ch.done != nullptr;
+  if (side) cudaStreamSynchronize(g->side);       // chunks still in flight there
   for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) dfree(g, *b);
-  for (auto &ch : p.chunks) dfree(g, ch.keys);
+  for (auto &ch : p.chunks) {
+    dfree(g, ch.keys);
+    dfree(g, ch.ctr);
+    if (ch.done) cudaEventDestroy(ch.done);
+  }
   p = PassOut();
 }
 
@@ -263,7 +270,36 @@ int64_t avail_bytes(sg_graph *g) {
 // computes each chunk's keys right before grouping it.
 double scratch_per_pair(int64_t maxseg);
 
-void plan_pass(sg_graph *g, PassOut &P) {
+void plan_pass_uncached(sg_graph *g, PassOut &P);
+
+// Memoised plan: same level, rows, trials and allocation state as a previous
+// step (single rank; multi-rank plans agree across ranks through a
+// collective, so they are always recomputed).
+void plan_pass(sg_graph *g, PassOut &P, int level) {
+  auto &m = g->plan_memo[level];
+  if (g->world == 1 && m.nrows == P.nrows && m.c == P.c && m.live == g->bytes_live &&
+      m.cached == g->bytes_cached) {
+    P.deferred = m.deferred;
+    P.chunks.clear();
+    for (auto &tc : m.chunks) {
+      KeyChunk k;
+      k.t0 = tc.first;
+      k.nt = tc.second;
+      P.chunks.push_back(k);
+    }
+    return;
+  }
+  m.live = g->bytes_live;
+  m.cached = g->bytes_cached;
+  plan_pass_uncached(g, P);
+  m.nrows = P.nrows;
+  m.c = P.c;
+  m.deferred = P.deferred;
+  m.chunks.clear();
+  for (auto &k : P.chunks) m.chunks.push_back({k.t0, k.nt});
+}
+
+void plan_pass_uncached(sg_graph *g, PassOut &P) {
   const int64_t nr = P.nrows, c = P.c;
   const double keys_t = 8.0 * (double)P.key_stride;             // keys of one trial
   const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;   // scratch per trial
@@ -305,12 +341,23 @@ void plan_pass(sg_graph *g, PassOut &P) {
   }
 }
 
-void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
-  st_begin(g, st_hash);
+// on_side: enqueue the kernels on the side stream after the buffers are
+// allocated in main-stream order; group_by_shingle waits on ch.done (the
+// chunk's keys and counters stay owned by the chunk until then).
+void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_side = false) {
+  if (!on_side) st_begin(g, st_hash);   // side chunks: timed on the side stream below
   dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
-  DBuf ctr;
+  DBuf &ctr = ch.ctr;
   dalloc(g, ctr, 16);
   CK(cudaMemsetAsync(ctr.p, 0, 16, g->stream));
+  cudaStream_t st = g->stream;
+  if (on_side) {
+    if (!ch.done) CK(cudaEventCreateWithFlags(&ch.done, cudaEventDisableTiming));
+    CK(cudaEventRecord(ch.done, g->stream));          // buffers ready (main-stream order)
+    CK(cudaStreamWaitEvent(g->side, ch.done, 0));
+    st = g->side;
+    st_begin(g, st_hash, st);
+  }
   MinhashArgs a;
   a.rstart = ptr<int64_t>(P.rstart);
   a.rlen = ptr<int32_t>(P.rlen);
@@ -327,9 +374,14 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash) {
   a.counter = ptr<unsigned long long>(ctr);
   a.hub_counter = a.counter + 1;
   a.tile_rows = st_hash == kStHash2 ? 16 : 8;   // pass II rows are short
-  CK(minhash(a, g->num_sms, g->stream));
-  dfree(g, ctr);
-  st_end(g, st_hash);
+  CK(minhash(a, g->num_sms, st));
+  if (on_side) {
+    st_end(g, st_hash, st);
+    CK(cudaEventRecord(ch.done, g->side));
+  } else {
+    dfree(g, ctr);
+    st_end(g, st_hash);
+  }
   ch.computed = true;
 }
 
@@ -892,6 +944,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
       CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
       g->own_stream = true;
     }
+    CK(cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking));
     // keep freed blocks cached in the pool: re-runs and resets reuse them
     cudaMemPool_t pool;
     CK(cudaDeviceGetDefaultMemPool(&pool, g->device));
@@ -953,6 +1006,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
     }
     cudaGetLastError();
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+    if (g->side) cudaStreamDestroy(g->side);
     return st;
   }
   *out = G.release();
@@ -1034,10 +1088,18 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     st_end(g, level == 0 ? kStSelect1 : kStSelect2);
     hm("select write enqueued");
     // ---- min-hash top-s of every row and trial (the hot kernel)
-    plan_pass(g, P);
+    plan_pass(g, P, level);
     hm("plan_pass");
-    if (!P.deferred)
-      for (auto &ch : P.chunks) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+    if (!P.deferred) {
+      // SG_OVERLAP=1 (experiment, off by default): chunk 0 on the main
+      // stream, the others on the side stream, overlapping the grouping of
+      // earlier chunks.  Measured on gos2m: 385.4 vs 381.6 ms serialised —
+      // the ALU-bound min-hash and the sort kernels contend for issue slots
+      // (hist2 doubles), so the default stays serial.
+      const bool overlap = g->side && g->world == 1 && P.chunks.size() > 1 && getenv("SG_OVERLAP");
+      for (size_t i = 0; i < P.chunks.size(); ++i)
+        compute_chunk(g, P, P.chunks[i], level == 0 ? kStHash1 : kStHash2, overlap && i > 0);
+    }
     hm("min-hash enqueued");
     st_end(g, st_all);
     sync(g);
@@ -1072,6 +1134,12 @@ sg_status group_by_shingle(sg_graph *g) {
       GroupScratch S;
       for (auto &ch : P.chunks) {
         if (!ch.computed) compute_chunk(g, P, ch, level == 0 ? kStHash1 : kStHash2);
+        if (ch.done) {
+          CK(cudaStreamWaitEvent(g->stream, ch.done, 0));   // keys computed on the side stream
+          cudaEventDestroy(ch.done);
+          ch.done = nullptr;
+          dfree(g, ch.ctr);
+        }
         std::vector<Piece> pieces;
         for (int tl = 0; tl < ch.nt; ++tl)
           pieces.push_back(Piece{tl, (int64_t)tl * P.key_stride, P.nrows, 0});
@@ -1107,6 +1175,7 @@ sg_status shingle_graph_reset(sg_graph *g) {
 void shingle_graph_destroy(sg_graph *g) {
   if (!g) return;
   cudaSetDevice(g->device);
+  if (g->side) cudaStreamSynchronize(g->side);   // side-stream chunks use the buffers below
   // stream-ordered frees back into the pool (cudaFree on pool blocks leaves
   // them accounted as used), then let the pool return them to the device
   auto rel = [&](void *p) {
@@ -1115,15 +1184,23 @@ void shingle_graph_destroy(sg_graph *g) {
   for (int l = 0; l < 2; ++l) {
     PassOut &p = g->pass[l];
     for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) rel(b->p);
-    for (auto &ch : p.chunks) rel(ch.keys.p);
+    for (auto &ch : p.chunks) {
+      rel(ch.keys.p);
+      rel(ch.ctr.p);
+    }
     for (DBuf *b : {&g->grp[l].members, &g->grp[l].head, &g->grp[l].okeys}) rel(b->p);
   }
   for (DBuf *b : {&g->row_ptr, &g->col}) rel(b->p);
   for (auto &c : g->cache) rel(c.p);
+  if (g->side) cudaStreamSynchronize(g->side);
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (cudaEvent_t e : g->ev_pool) cudaEventDestroy(e);
+  for (int l = 0; l < 2; ++l)
+    for (auto &ch : g->pass[l].chunks)
+      if (ch.done) cudaEventDestroy(ch.done);
   if (g->xch) exchange_destroy(g->xch);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+  if (g->side) cudaStreamDestroy(g->side);
   cudaGetLastError();
   delete g;
 }

@@ -80,6 +80,8 @@ struct KeyChunk {
   int32_t t0 = 0, nt = 0;
   bool computed = false;
   DBuf keys;
+  DBuf ctr;                        // the min-hash tile counters (kept while in flight)
+  cudaEvent_t done = nullptr;      // recorded on the side stream when computed there
 };
 
 // One shingling pass on this rank.
@@ -139,6 +141,7 @@ struct sg_graph {
   int32_t device = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  cudaStream_t side = nullptr;     // min-hash of later trial chunks, overlapped with grouping
   int32_t rank = 0, world = 1;
   sg::Exchange *xch = nullptr;
   int num_sms = 148;
@@ -163,6 +166,14 @@ struct sg_graph {
   std::vector<std::pair<int, int>> st[sg::kNumStages];
   int64_t mem_budget = 0;       // test hook: cap on planned bytes (0 = free HBM)
   int64_t bytes_live = 0;       // device bytes currently held by this handle
+  // plan_pass memo per level: the device memory query (cudaMemGetInfo) can
+  // take milliseconds under load, and repeated steps plan the same pass in
+  // the same allocation state
+  struct PlanMemo {
+    int64_t nrows = -1, c = -1, live = -1, cached = -1;
+    bool deferred = false;
+    std::vector<std::pair<int32_t, int32_t>> chunks;
+  } plan_memo[2];
   std::vector<sg::DBuf> cache;  // freed blocks kept for reuse (best fit)
   int64_t bytes_cached = 0;
 };
