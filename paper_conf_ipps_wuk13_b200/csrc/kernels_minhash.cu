@@ -140,27 +140,24 @@ __device__ __forceinline__ uint32_t hash_or_pad(uint32_t A, uint32_t B, uint32_t
   return m31_hash(A, B, v) | (uint32_t)((int32_t)v >> 31);
 }
 
-// Two rows of QA / QB padded quads, scanned side by side (independent chains).
-template <int S, int QA, int QB>
-__device__ __forceinline__ void quads2(const uint32_t *pa, const uint32_t *pb, uint32_t A,
-                                       uint32_t B, uint32_t (&ma)[S], uint32_t (&mb)[S]) {
-  const uint4 *a4 = reinterpret_cast<const uint4 *>(pa);
-  const uint4 *b4 = reinterpret_cast<const uint4 *>(pb);
+// Two rows of na / nb (<= 4, warp-uniform) padded pairs, scanned side by
+// side: 64-bit broadcast loads, so a 2-entry row hashes 2 slots, not 4.
+template <int S>
+__device__ __forceinline__ void pairs2(const uint32_t *pa, const uint32_t *pb, int na, int nb,
+                                       uint32_t A, uint32_t B, uint32_t (&ma)[S], uint32_t (&mb)[S]) {
+  const uint2 *a2 = reinterpret_cast<const uint2 *>(pa);
+  const uint2 *b2 = reinterpret_cast<const uint2 *>(pb);
 #pragma unroll
-  for (int q = 0; q < (QA > QB ? QA : QB); ++q) {
-    if (q < QA) {
-      const uint4 v = a4[q];
+  for (int q = 0; q < 4; ++q) {
+    if (q < na) {
+      const uint2 v = a2[q];
       insert_min<S>(ma, hash_or_pad(A, B, v.x));
       insert_min<S>(ma, hash_or_pad(A, B, v.y));
-      insert_min<S>(ma, hash_or_pad(A, B, v.z));
-      insert_min<S>(ma, hash_or_pad(A, B, v.w));
     }
-    if (q < QB) {
-      const uint4 v = b4[q];
+    if (q < nb) {
+      const uint2 v = b2[q];
       insert_min<S>(mb, hash_or_pad(A, B, v.x));
       insert_min<S>(mb, hash_or_pad(A, B, v.y));
-      insert_min<S>(mb, hash_or_pad(A, B, v.z));
-      insert_min<S>(mb, hash_or_pad(A, B, v.w));
     }
   }
 }
@@ -303,12 +300,7 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
               uint32_t ma[S], mb[S];
 #pragma unroll
               for (int i = 0; i < S; ++i) ma[i] = mb[i] = 0xFFFFFFFFu;
-              switch ((la > 4) * 2 + (lb > 4)) {
-                case 0: quads2<S, 1, 1>(pa, pb, A, B, ma, mb); break;
-                case 1: quads2<S, 1, 2>(pa, pb, A, B, ma, mb); break;
-                case 2: quads2<S, 2, 1>(pa, pb, A, B, ma, mb); break;
-                default: quads2<S, 2, 2>(pa, pb, A, B, ma, mb); break;
-              }
+              pairs2<S>(pa, pb, (la + 1) >> 1, (lb + 1) >> 1, A, B, ma, mb);
               sOut[out_slot(rr, lane)] = fmix(shingle_id<S>(ma, a.seed, a.t0 + j));
               sOut[out_slot(rr + 1, lane)] = fmix(shingle_id<S>(mb, a.seed, a.t0 + j));
               rr += 2;
