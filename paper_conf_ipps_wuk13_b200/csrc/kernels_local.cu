@@ -82,6 +82,7 @@ constexpr int kWBatch = kWCap / 32;        // 32 batches of 32 positions
 constexpr int kWWarps = 7;                 // warps per CTA (3 CTAs, 21 warps per SM)
 constexpr int kWDigitBits = 10;            // two LSD passes = 20 key bits
 constexpr int kWDigits = 1 << kWDigitBits;
+constexpr int kWB = 8;                     // batches of 32 in flight (placement, emit)
 
 struct __align__(16) WarpSmem {
   uint32_t d20[kWCap];        // the 20 key bits after the bucket bits
@@ -123,10 +124,10 @@ __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint1
   const int lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   uint32_t *cw = reinterpret_cast<uint32_t *>(cur);
-  for (int i0 = 0; i0 < n; i0 += 128) {
-    uint32_t e[4], d[4], m[4], o[4];
+  for (int i0 = 0; i0 < n; i0 += 32 * kWB) {
+    uint32_t e[kWB], d[kWB], m[kWB], o[kWB];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kWB; ++u) {
       const int i = i0 + u * 32 + lane;
       const bool valid = i < n;
       e[u] = valid ? (FIRST ? (uint32_t)i : (uint32_t)src[i]) : 0u;
@@ -137,7 +138,7 @@ __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint1
         o[u] = atomicAdd(&cw[d[u] >> 1], (uint32_t)__popc(m[u]) << ((d[u] & 1) << 4));
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kWB; ++u) {
       const uint32_t oo = __shfl_sync(0xffffffffu, o[u], __ffs(m[u]) - 1);
       if (i0 + u * 32 + lane < n) {
         const uint32_t base = (oo >> ((d[u] & 1) << 4)) & 0xFFFFu;
@@ -157,23 +158,23 @@ __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n
   const int lane = threadIdx.x & 31;
   bool bad = false;
   uint64_t carry = 0;
-  for (int p0 = 0; p0 < n; p0 += 128) {
-    int e[4];
-    uint64_t ke[4];
-    uint32_t ve[4];
+  for (int p0 = 0; p0 < n; p0 += 32 * kWB) {
+    int e[kWB];
+    uint64_t ke[kWB];
+    uint32_t ve[kWB];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kWB; ++u) {
       const int p = p0 + u * 32 + lane;
       e[u] = p < n ? pm[p] : 0;
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kWB; ++u) {
       const bool valid = p0 + u * 32 + lane < n;
       ke[u] = valid ? Kg[e[u]] : ~0ull;
       ve[u] = valid ? Vg[e[u]] : 0u;
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kWB; ++u) {
       if (p0 + u * 32 >= n) break;                    // warp-uniform
       const int p = p0 + u * 32 + lane;
       const bool valid = p < n;
@@ -194,7 +195,7 @@ __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n
   return __any_sync(0xffffffffu, bad);
 }
 
-__global__ void __launch_bounds__(kWWarps * 32) warp_local_kernel(const __grid_constant__ GroupArgs g) {
+__global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   WarpSmem &S = reinterpret_cast<WarpSmem *>(smraw)[wl];
