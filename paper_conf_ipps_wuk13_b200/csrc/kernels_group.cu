@@ -332,7 +332,18 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   // fine-bucket totals (order-free), starts, sizes
   for (int i = threadIdx.x; i < nb2; i += blockDim.x) S.tot[i] = 0;
   __syncthreads();
-  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&S.tot[fine(K[i])], 1u);
+  {
+    // four loads in flight per thread
+    int64_t i = threadIdx.x;
+    for (; i + 3 * kSThreads < n; i += 4 * kSThreads) {
+      const uint64_t k0 = K[i], k1 = K[i + kSThreads], k2 = K[i + 2 * kSThreads], k3 = K[i + 3 * kSThreads];
+      atomicAdd(&S.tot[fine(k0)], 1u);
+      atomicAdd(&S.tot[fine(k1)], 1u);
+      atomicAdd(&S.tot[fine(k2)], 1u);
+      atomicAdd(&S.tot[fine(k3)], 1u);
+    }
+    for (; i < n; i += kSThreads) atomicAdd(&S.tot[fine(K[i])], 1u);
+  }
   __syncthreads();
   {
     const int d = threadIdx.x;
