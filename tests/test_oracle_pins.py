@@ -356,3 +356,80 @@ def test_report_labels_are_min_of_class():
         classes[l].append(v)
     assert all(min(vs) == l for l, vs in classes.items())
     assert nc == sum(1 for vs in classes.values() if len(vs) >= 2)
+
+
+# ---------------------------------------------------------------- Phase III approach 1
+@pytest.mark.parametrize("mode", [0, 1])
+def test_overlapping_planted_cliques_exact(mode):
+    """Disjoint planted cliques: approach 1 reports exactly the cliques."""
+    sizes = [5, 6, 8, 10, 12, 15, 20, 25, 30, 9, 7, 11]
+    g = SG.cliques(sizes, n=sum(sizes) + 40, seed=17)
+    res = oracle.shingling(g.row_ptr, g.col, 2, 100, 21, 2, 100, 22)
+    offs, verts = oracle.report_overlapping(res, g.row_ptr, g.col, mode)
+    got = sorted(tuple(verts[offs[i]:offs[i + 1]].tolist()) for i in range(len(offs) - 1))
+    deg = g.degrees()
+    comp = _components(g)
+    by_comp = defaultdict(list)
+    for v in range(g.n):
+        if deg[v] > 0:
+            by_comp[comp[v]].append(v)
+    assert got == sorted(tuple(sorted(x)) for x in by_comp.values())
+
+
+@pytest.mark.parametrize("s1,gseed", [(1, 6), (2, 7), (2, 8)])
+def test_overlapping_equals_decoded_bfs(s1, gseed):
+    """Brute force: constituents decoded algebraically from the exact ids
+    (v = (h - B_j) A_j^(P-2) mod P, s <= 2, AMB-4), components by a plain BFS
+    over G_II groups (every group joins all its members)."""
+    g = SG.Graph(*SG.homology_graph(n=300, n_isolated=20, m_target=2500, seed=gseed, n_cliques=3,
+                                    clique_lo=6, clique_hi=12, cc_max=120, fam_hi=40))
+    res = oracle.shingling(g.row_ptr, g.col, s1, 12, 100 + gseed, 2, 8, 200 + gseed)
+    nk = len(res.s1p_group)
+    assert nk > 0
+    adj = defaultdict(set)
+    G2 = res.G2
+    for gi in range(len(G2.ids)):
+        K = G2.members[G2.offs[gi]:G2.offs[gi + 1]].tolist()
+        for x in K:
+            adj[x].update(K)
+    tg1 = res.G1.trial_goffs.tolist()
+
+    def decode(gi):
+        j = max(t for t in range(len(tg1) - 1) if tg1[t] <= gi)
+        idv = int(res.G1.ids[gi])
+        hs = [idv] if s1 == 1 else [idv >> 31, idv & P]
+        A, B = int(res.A1[j]), int(res.B1[j])
+        return {((h - B) * pow(A, P - 2, P)) % P for h in hs}
+
+    seen = [False] * nk
+    want = []
+    for k0 in range(nk):
+        if seen[k0]:
+            continue
+        seen[k0] = True
+        stack, S = [k0], set()
+        while stack:
+            k = stack.pop()
+            S |= decode(int(res.s1p_group[k]))
+            for y in adj[k]:
+                if not seen[y]:
+                    seen[y] = True
+                    stack.append(y)
+        want.append(sorted(S))
+    for ms in (1, 4):
+        offs, verts = oracle.report_overlapping(res, g.row_ptr, g.col, 0, ms)
+        got = [verts[offs[i]:offs[i + 1]].tolist() for i in range(len(offs) - 1)]
+        assert got == [w for w in want if len(w) >= ms]
+
+
+def test_overlapping_inside_union_find_clusters():
+    """Each approach-1 cluster lies inside one approach-2 cluster (approach 2
+    unions a superset of the same constituents)."""
+    g = SG.Graph(*SG.homology_graph(n=300, n_isolated=20, m_target=2500, seed=9, n_cliques=3,
+                                    clique_lo=6, clique_hi=12, cc_max=120, fam_hi=40))
+    res = oracle.shingling(g.row_ptr, g.col, 2, 16, 109, 2, 12, 209)
+    labels, _ = res.report(mode=0)
+    offs, verts = oracle.report_overlapping(res, g.row_ptr, g.col, 0)
+    assert len(offs) > 1
+    for i in range(len(offs) - 1):
+        assert len(set(labels[verts[offs[i]:offs[i + 1]]].tolist())) == 1
