@@ -132,6 +132,29 @@ SG_API sg_status group_by_shingle(sg_graph *g);
 SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
                                  int64_t *n_clusters);
 
+/* ------------------------------------------------------------------------ */
+/* report_overlapping_clusters — Phase III, approach 1:        */
+/* "enumerate all connected components in G_II ... for each connected      */
+/* component, report the set of all vertices in G that constitute the       */
+/* first-level shingles of that component as a cluster" (clusters may       */
+/* overlap).  Components join S1' nodes through shared G_II groups.         */
+/*   mode     0: constituents (top-s1 vertices of the smallest generator's  */
+/*            row under H1[j], AMB-9/AMB-18); 1: the generators L(s).       */
+/*   min_size clusters with fewer vertices are not reported.                */
+/*   offs     host int64[C+1], verts host uint32[V]: cluster i is            */
+/*            verts[offs[i], offs[i+1]), vertices ascending; clusters in     */
+/*            order of their smallest S1' index.  Caller-allocated; caps =   */
+/*            {C+1, V}.  Both NULL: only counts <- {C, V} (two-call pattern; */
+/*            each call recomputes on the device).                          */
+/* Union-find over S1', constituent emission, radix sort + unique on the    */
+/* device; the host splits the sorted list.  Untimed; state GROUPED2,       */
+/* world == 1.  Errors: SG_EINVAL (mode, NULL counts, caps too small),      */
+/* SG_ESTATE, SG_ENOMEM, SG_ECUDA, SG_EOVERFLOW (> 2^31 constituents).      */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_size,
+                                             int64_t *offs, uint32_t *verts, const int64_t caps[2],
+                                             int64_t counts[2]);
+
 /* Return the handle to state CREATED (CSR kept, results dropped) so the two */
 /* passes can be run again, e.g. by a benchmark.                             */
 SG_API sg_status shingle_graph_reset(sg_graph *g);

@@ -57,6 +57,7 @@ def lib() -> C.CDLL:
         "shingle_pass": (st, [vp, i32, i32, u64]),
         "group_by_shingle": (st, [vp]),
         "report_dense_subgraphs": (st, [vp, i32, i32, vp, vp]),
+        "report_overlapping_clusters": (st, [vp, i32, i32, vp, vp, vp, vp]),
         "shingle_graph_reset": (st, [vp]),
         "shingle_graph_destroy": (None, [vp]),
         "sg_last_error": (C.c_char_p, [vp]),
@@ -138,6 +139,18 @@ def report_dense_subgraphs(h, mode: int = 0, min_size: int = 1, n: Optional[int]
     nc = C.c_int64()
     _check(lib().report_dense_subgraphs(h, mode, min_size, labels.ctypes.data, C.byref(nc)), h)
     return labels, nc.value
+
+
+def report_overlapping_clusters(h, mode: int = 0, min_size: int = 1):
+    """Phase III approach 1: (offs int64[C+1], verts uint32[V])."""
+    cnt = np.zeros(2, np.int64)
+    _check(lib().report_overlapping_clusters(h, mode, min_size, None, None, None, cnt.ctypes.data), h)
+    offs = np.zeros(int(cnt[0]) + 1, np.int64)
+    verts = np.zeros(int(cnt[1]), np.uint32)
+    caps = np.array([len(offs), len(verts)], np.int64)
+    _check(lib().report_overlapping_clusters(h, mode, min_size, offs.ctypes.data, verts.ctypes.data,
+                                             caps.ctypes.data, cnt.ctypes.data), h)
+    return offs, verts
 
 
 def shingle_graph_reset(h):
@@ -263,6 +276,9 @@ class ShingleGraph:
 
     def report(self, mode=0, min_size=1):
         return report_dense_subgraphs(self.h, mode, min_size, self.n)
+
+    def report_overlapping(self, mode=0, min_size=1):
+        return report_overlapping_clusters(self.h, mode, min_size)
 
     def reset(self):
         shingle_graph_reset(self.h)

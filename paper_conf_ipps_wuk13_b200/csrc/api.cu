@@ -1487,4 +1487,91 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
   });
 }
 
+sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_size, int64_t *offs,
+                                      uint32_t *verts, const int64_t caps[2], int64_t counts[2]) {
+  return guarded(g, [&] {
+    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
+    if (!counts) fail(g, SG_EINVAL, "counts is NULL");
+    if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
+    if (g->world > 1) require_single(g, "report_overlapping_clusters");
+    PassOut &P1 = g->pass[0];
+    PassOut &P2 = g->pass[1];
+    ReportArgs a;
+    a.n = g->n;
+    a.mode = mode;
+    a.min_size = min_size;
+    a.s1 = P1.s;
+    a.s2 = P2.s;
+    a.A1 = ptr<uint32_t>(P1.A);
+    a.B1 = ptr<uint32_t>(P1.B);
+    a.row_ptr = ptr<int64_t>(g->row_ptr);
+    a.col = ptr<uint32_t>(g->col);
+    a.members1 = ptr<uint32_t>(g->grp[0].members);
+    a.rows1 = P1.nrows;
+    a.rstart2 = ptr<int64_t>(P2.rstart);
+    a.rlen2 = ptr<int32_t>(P2.rlen);
+    a.nk = P2.nrows;
+    a.members2 = ptr<uint32_t>(g->grp[1].members);
+    a.head2 = ptr<uint32_t>(g->grp[1].head);
+    a.npairs2 = g->grp[1].npairs;
+    a.rows2 = P2.nrows;
+    DBuf parentK, eoff, keys, sorted, temp, dn;
+    dalloc(g, dn, 8);
+    int64_t nkeys = a.nk * (int64_t)a.s1;
+    if (mode == 1) {
+      unsigned long long e2 = 0;
+      CK(sum_i32(a.rlen2, a.nk, ptr<unsigned long long>(dn), g->stream));
+      CK(cudaMemcpyAsync(&e2, dn.p, 8, cudaMemcpyDeviceToHost, g->stream));
+      sync(g);
+      nkeys = (int64_t)e2;
+    }
+    if (nkeys > INT32_MAX || a.nk > INT32_MAX)
+      fail(g, SG_EOVERFLOW, "report_overlapping_clusters: more than 2^31 constituents");
+    const size_t tb = overlap_temp_bytes(a.nk, nkeys);
+    dalloc(g, parentK, (size_t)a.nk * 4);
+    dalloc(g, eoff, (size_t)a.nk * 8);
+    dalloc(g, keys, (size_t)nkeys * 8);
+    dalloc(g, sorted, (size_t)nkeys * 8);
+    dalloc(g, temp, tb);
+    CK(overlap_device(a, ptr<uint32_t>(parentK), ptr<int64_t>(eoff), ptr<uint64_t>(keys),
+                      ptr<uint64_t>(sorted), nkeys, temp.p, temp.bytes, ptr<int64_t>(dn),
+                      g->num_sms, g->stream));
+    int64_t nu = 0;
+    CK(cudaMemcpyAsync(&nu, dn.p, 8, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    std::vector<uint64_t> u((size_t)nu);
+    if (nu) CK(cudaMemcpyAsync(u.data(), keys.p, (size_t)nu * 8, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    for (DBuf *b : {&parentK, &eoff, &keys, &sorted, &temp, &dn}) dfree(g, *b);
+    if (nu && u[(size_t)nu - 1] == ~0ull) --nu;         // rows shorter than s1 (none in practice)
+    // split the sorted (root, vertex) list into clusters; drop the small ones
+    const int64_t thr = std::max<int32_t>(1, min_size);
+    int64_t nc = 0, nv = 0;
+    for (int64_t i = 0; i < nu;) {
+      int64_t e = i + 1;
+      while (e < nu && (u[(size_t)e] >> 32) == (u[(size_t)i] >> 32)) ++e;
+      if (e - i >= thr) {
+        if (offs || verts) {
+          if (!caps || caps[0] < nc + 2 || caps[1] < nv + (e - i)) fail(g, SG_EINVAL, "buffers too small");
+          if (offs) {
+            offs[nc] = nv;
+            offs[nc + 1] = nv + (e - i);
+          }
+          if (verts)
+            for (int64_t x = i; x < e; ++x) verts[nv + (x - i)] = (uint32_t)u[(size_t)x];
+        }
+        ++nc;
+        nv += e - i;
+      }
+      i = e;
+    }
+    if (offs && nc == 0) {
+      if (!caps || caps[0] < 1) fail(g, SG_EINVAL, "buffers too small");
+      offs[0] = 0;
+    }
+    counts[0] = nc;
+    counts[1] = nv;
+  });
+}
+
 }  // extern "C"

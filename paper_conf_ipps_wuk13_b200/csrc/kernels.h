@@ -151,6 +151,15 @@ struct ReportArgs {
 cudaError_t report_device(const ReportArgs &a, uint32_t *parent, uint32_t *rep1, uint32_t *size,
                           int32_t *labels, unsigned long long *d_nc, int num_sms, cudaStream_t st);
 
+// Phase III approach 1 (overlapping clusters): parentK uint32[nk]; eoff
+// int64[nk] (mode 1); keys / keys_sorted uint64[nkeys] (mode 0: nk * s1, mode
+// 1: sum of |L(k)|); afterwards keys[0, *d_nuniq) = sorted unique
+// (component root << 32 | vertex), sentinels ~0 last.
+size_t overlap_temp_bytes(int64_t nk, int64_t nkeys);
+cudaError_t overlap_device(const ReportArgs &a, uint32_t *parentK, int64_t *eoff, uint64_t *keys,
+                           uint64_t *keys_sorted, int64_t nkeys, void *temp, size_t temp_bytes,
+                           int64_t *d_nuniq, int num_sms, cudaStream_t st);
+
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);

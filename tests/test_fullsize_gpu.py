@@ -43,7 +43,8 @@ def run():
     B.shingle_pass(h, cfg["s2"], cfg["c2"], cfg["seed2"])
     B.group_by_shingle(h)
     out = dict(counts=B.sg_get_counts(h), M1=B.sg_get_shingles(h, 1), G1=B.sg_get_groups(h, 1),
-               s1p=B.sg_get_s1p(h), A1=B.sg_get_hash_params(h, 1, cfg["c1"]))
+               s1p=B.sg_get_s1p(h), A1=B.sg_get_hash_params(h, 1, cfg["c1"]),
+               rep0=B.report_dense_subgraphs(h, 0, 1, g.n), ov=B.report_overlapping_clusters(h, 0))
     B.shingle_graph_destroy(h)
     return g, cfg, out
 
@@ -103,3 +104,36 @@ def test_fullsize_s1p_filter_and_level2_counts(run):
     assert c["entries2"] == int(sizes[sel].sum())
     assert c["pairs2"] == len(sel) * cfg["c2"]
     assert len(sel) <= c["groups2"] <= c["pairs2"]
+
+
+def test_fullsize_overlapping_clusters(run):
+    """Phase III approach 1 at full size: clusters are ascending
+    vertex lists, each inside one approach-2 cluster (P:L483-488 unions a
+    superset of the same constituents); sampled S1' nodes' constituents,
+    recomputed one by one by the oracle, appear among the clustered vertices."""
+    g, cfg, out = run
+    offs, verts = out["ov"]
+    labels, _ = out["rep0"]
+    C = len(offs) - 1
+    assert C > 0 and offs[0] == 0 and offs[-1] == len(verts)
+    sizes = np.diff(offs)
+    assert sizes.min() >= 1
+    v = verts.astype(np.int64)
+    inner = np.ones(len(v), bool)
+    inner[offs[:-1]] = False
+    assert np.all(v[1:][inner[1:]] > v[:-1][inner[1:]])          # ascending within a cluster
+    lab = labels[v].astype(np.int64)
+    assert np.array_equal(np.minimum.reduceat(lab, offs[:-1]), np.maximum.reduceat(lab, offs[:-1]))
+    clustered = np.zeros(g.n, bool)
+    clustered[v] = True
+    tg, gid, goffs, mem = out["G1"]
+    A, Bv = out["A1"]
+    s1p, _ = out["s1p"]
+    rng = np.random.default_rng(5)
+    for k in rng.choice(len(s1p), 200, replace=False):
+        gi = int(s1p[k])
+        j = int(np.searchsorted(tg, gi, side="right") - 1)
+        u = int(mem[goffs[gi]])
+        row = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
+        cons = oracle.row_constituents(row, cfg["s1"], int(A[j]), int(Bv[j]))
+        assert clustered[cons].all()

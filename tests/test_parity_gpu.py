@@ -224,3 +224,56 @@ def test_invalid_csr_rejected(B):
         with pytest.raises(B.SGError) as e:
             B.shingle_graph_create(rp, col)
         assert e.value.status == B.SG_EINVAL
+
+
+# ---------------------------------------------------------------- Phase III approach 1
+def _ov_case(B, g, s1, c1, seed1, s2, c2, seed2, modes=(0, 1), sizes=(1, 3)):
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        G.run(s1, c1, seed1, s2, c2, seed2)
+        got = {(m, ms): G.report_overlapping(m, ms) for m in modes for ms in sizes}
+    ref = oracle.shingling(g.row_ptr, g.col, s1, c1, seed1, s2, c2, seed2)
+    for (m, ms), (offs, verts) in got.items():
+        ro, rv = oracle.report_overlapping(ref, g.row_ptr, g.col, m, ms)
+        assert np.array_equal(offs, ro), (m, ms)
+        assert np.array_equal(verts, rv), (m, ms)
+    return got
+
+
+def test_overlapping_tiny_config(B):
+    """BASELINE configs[0] (10K vertices, 50 planted cliques, s=2, c=100)."""
+    g = SG.make("tiny")
+    cfg = SG.CONFIGS["tiny"]
+    got = _ov_case(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
+                   sizes=(1, 20))
+    assert len(got[(0, 20)][0]) - 1 >= 50
+
+
+@pytest.mark.parametrize("s1,c1,s2,c2,gseed", [(1, 20, 1, 9, 31), (2, 33, 2, 40, 32),
+                                             (3, 24, 2, 17, 33), (4, 40, 3, 33, 34)])
+def test_overlapping_small_graphs(B, s1, c1, s2, c2, gseed):
+    g = SG.Graph(*SG.homology_graph(n=3000, n_isolated=300, m_target=40000, seed=gseed,
+                                    n_cliques=12, clique_lo=6, clique_hi=30, cc_max=600,
+                                    fam_hi=200))
+    _ov_case(B, g, s1, c1, 100 + gseed, s2, c2, 200 + gseed)
+
+
+def test_overlapping_planted_cliques_and_empty(B):
+    sizes = [5, 6, 8, 10, 12, 15, 20, 25, 30, 9, 7, 11]
+    g = SG.cliques(sizes, n=sum(sizes) + 40, seed=17)
+    got = _ov_case(B, g, 2, 100, 21, 2, 100, 22)
+    assert len(got[(0, 1)][0]) - 1 == len(sizes)
+    # no first-level group reaches s2 -> no S1' node, no cluster
+    g3 = SG.cliques([3, 3, 3], n=20, seed=3)
+    got = _ov_case(B, g3, 2, 16, 5, 2, 16, 6)
+    for offs, verts in got.values():
+        assert len(offs) == 1 and len(verts) == 0
+
+
+def test_overlapping_errors(B):
+    g = SG.cliques([6, 7], n=20, seed=4)
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        with pytest.raises(B.SGError):
+            G.report_overlapping(0)          # not grouped yet
+        G.run(2, 8, 1, 2, 8, 2)
+        with pytest.raises(B.SGError):
+            G.report_overlapping(2)          # bad mode
