@@ -256,6 +256,13 @@ def bench_ours(args, rank, world, local_rank):
         _, ncl = B.report_dense_subgraphs(h, 0, 20, g.n)
         phase3 = {"ms": round(B.sg_get_stage_ms(h).get("report", 0.0), 3), "clusters_ge20": int(ncl),
                   "mode": "constituents (AMB-9)", "timed_in_metric": False}
+        # approach 1 (overlapping clusters), host-timed: both calls of
+        # the two-call pattern (sizes, then fill), each recomputing on the device
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        ooffs, _ = B.report_overlapping_clusters(h, 0, 20)
+        phase3["overlapping"] = {"ms_host": round((time.perf_counter() - t0) * 1e3, 3),
+                                 "clusters_ge20": int(len(ooffs) - 1)}
     B.shingle_graph_destroy(h)
 
     # ---- e2e: the public API with host buffers, H2D + D2H inside the region
