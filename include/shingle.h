@@ -155,6 +155,24 @@ SG_API sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t 
                                              int64_t *offs, uint32_t *verts, const int64_t caps[2],
                                              int64_t counts[2]);
 
+/* ------------------------------------------------------------------------ */
+/* sg_cluster_density — Eq. 6: density of a cluster =       */
+/* #(edges in the cluster) / #(possible edges) = e / C(k, 2), averaged over */
+/* the clusters of a partition (the paper: 0.75 +- 0.28 for gpClust on the  */
+/* 2M GOS graph, Table IV context).                                          */
+/*   labels   host int32[n], labels[v] in [0, n) names v's cluster (e.g. the */
+/*            output of report_dense_subgraphs); borrowed, copied to HBM.    */
+/*   min_size clusters with fewer than max(2, min_size) vertices are skipped.*/
+/*   mean, stddev (population) and n_clusters receive the statistics over    */
+/*   the counted clusters (0 when none); each may be NULL.                   */
+/* Intra-cluster edges are counted on the device (one warp per row, over   */
+/* the resident CSR; undirected edges are stored twice, AMB-11).  Any state */
+/* after create; world == 1.  Errors: SG_EINVAL (NULL labels, label out of  */
+/* range), SG_ESTATE, SG_ENOMEM, SG_ECUDA.                                   */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_size,
+                                    double *mean, double *stddev, int64_t *n_clusters);
+
 /* Return the handle to state CREATED (CSR kept, results dropped) so the two */
 /* passes can be run again, e.g. by a benchmark.                             */
 SG_API sg_status shingle_graph_reset(sg_graph *g);

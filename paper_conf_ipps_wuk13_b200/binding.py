@@ -58,6 +58,7 @@ def lib() -> C.CDLL:
         "group_by_shingle": (st, [vp]),
         "report_dense_subgraphs": (st, [vp, i32, i32, vp, vp]),
         "report_overlapping_clusters": (st, [vp, i32, i32, vp, vp, vp, vp]),
+        "sg_cluster_density": (st, [vp, vp, i32, vp, vp, vp]),
         "shingle_graph_reset": (st, [vp]),
         "shingle_graph_destroy": (None, [vp]),
         "sg_last_error": (C.c_char_p, [vp]),
@@ -151,6 +152,15 @@ def report_overlapping_clusters(h, mode: int = 0, min_size: int = 1):
     _check(lib().report_overlapping_clusters(h, mode, min_size, offs.ctypes.data, verts.ctypes.data,
                                              caps.ctypes.data, cnt.ctypes.data), h)
     return offs, verts
+
+
+def sg_cluster_density(h, labels, min_size: int = 2):
+    """Eq. 6 density over the clusters of `labels`: (mean, stddev, n_clusters)."""
+    labels = np.ascontiguousarray(labels, np.int32)
+    mean, sd, nc = C.c_double(), C.c_double(), C.c_int64()
+    _check(lib().sg_cluster_density(h, labels.ctypes.data, min_size, C.byref(mean), C.byref(sd),
+                                    C.byref(nc)), h)
+    return mean.value, sd.value, nc.value
 
 
 def shingle_graph_reset(h):
@@ -276,6 +286,9 @@ class ShingleGraph:
 
     def report(self, mode=0, min_size=1):
         return report_dense_subgraphs(self.h, mode, min_size, self.n)
+
+    def density(self, labels, min_size=2):
+        return sg_cluster_density(self.h, labels, min_size)
 
     def report_overlapping(self, mode=0, min_size=1):
         return report_overlapping_clusters(self.h, mode, min_size)

@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -1571,6 +1572,47 @@ sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_siz
     }
     counts[0] = nc;
     counts[1] = nv;
+  });
+}
+
+sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_size, double *mean,
+                             double *stddev, int64_t *n_clusters) {
+  return guarded(g, [&] {
+    if (!labels) fail(g, SG_EINVAL, "labels is NULL");
+    if (g->world > 1) require_single(g, "sg_cluster_density");
+    if (g->state < kCreated) fail(g, SG_ESTATE, "no graph");
+    const int64_t n = g->n;
+    for (int64_t v = 0; v < n; ++v)
+      if (labels[v] < 0 || labels[v] >= n) fail(g, SG_EINVAL, "labels must lie in [0, n)");
+    DBuf dl, de, ds;
+    dalloc(g, dl, (size_t)n * 4);
+    dalloc(g, de, (size_t)n * 8);
+    dalloc(g, ds, (size_t)n * 4);
+    CK(cudaMemcpyAsync(dl.p, labels, (size_t)n * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(density_device(ptr<int64_t>(g->row_ptr), ptr<uint32_t>(g->col), n, ptr<int32_t>(dl),
+                      ptr<unsigned long long>(de), ptr<uint32_t>(ds), g->num_sms, g->stream));
+    std::vector<unsigned long long> e2((size_t)n);
+    std::vector<uint32_t> sz((size_t)n);
+    CK(cudaMemcpyAsync(e2.data(), de.p, (size_t)n * 8, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaMemcpyAsync(sz.data(), ds.p, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    for (DBuf *b : {&dl, &de, &ds}) dfree(g, *b);
+    // mean and population standard deviation over clusters of >= max(2, min_size)
+    const int64_t thr = std::max<int32_t>(2, min_size);
+    int64_t c = 0;
+    double s1 = 0.0, s2 = 0.0;
+    for (int64_t r = 0; r < n; ++r) {
+      const int64_t k = sz[(size_t)r];
+      if (k < thr) continue;
+      const double d = (double)(e2[(size_t)r] / 2) / ((double)k * (double)(k - 1) / 2.0);
+      ++c;
+      s1 += d;
+      s2 += d * d;
+    }
+    const double mu = c ? s1 / (double)c : 0.0;
+    if (mean) *mean = mu;
+    if (stddev) *stddev = c ? std::sqrt(std::max(0.0, s2 / (double)c - mu * mu)) : 0.0;
+    if (n_clusters) *n_clusters = c;
   });
 }
 

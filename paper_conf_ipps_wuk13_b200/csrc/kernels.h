@@ -160,6 +160,12 @@ cudaError_t overlap_device(const ReportArgs &a, uint32_t *parentK, int64_t *eoff
                            uint64_t *keys_sorted, int64_t nkeys, void *temp, size_t temp_bytes,
                            int64_t *d_nuniq, int num_sms, cudaStream_t st);
 
+// Cluster density (Eq. 6): e2[label] = 2 x intra-cluster edges, size[label] =
+// vertices, both device [n] and zeroed here; labels device int32[n] in [0, n).
+cudaError_t density_device(const int64_t *row_ptr, const uint32_t *col, int64_t n,
+                           const int32_t *labels, unsigned long long *e2, uint32_t *size,
+                           int num_sms, cudaStream_t st);
+
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);

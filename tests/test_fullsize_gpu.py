@@ -45,6 +45,17 @@ def run():
     out = dict(counts=B.sg_get_counts(h), M1=B.sg_get_shingles(h, 1), G1=B.sg_get_groups(h, 1),
                s1p=B.sg_get_s1p(h), A1=B.sg_get_hash_params(h, 1, cfg["c1"]),
                rep0=B.report_dense_subgraphs(h, 0, 1, g.n), ov=B.report_overlapping_clusters(h, 0))
+    # density (Eq. 6): all clusters >= 20, and a sample of 30 clusters (the
+    # rest relabelled as singletons) that the oracle recounts edge by edge
+    labels = out["rep0"][0]
+    out["nc20"] = B.report_dense_subgraphs(h, 0, 20, g.n)[1]
+    out["dens20"] = B.sg_cluster_density(h, labels, 20)
+    roots, sizes = np.unique(labels, return_counts=True)
+    cand = roots[(sizes >= 2) & (sizes <= 300)]
+    pick = np.random.default_rng(11).choice(cand, 30, replace=False)
+    lab_s = np.where(np.isin(labels, pick), labels, np.arange(g.n, dtype=np.int32)).astype(np.int32)
+    out["lab_s"] = lab_s
+    out["dens_s"] = B.sg_cluster_density(h, lab_s, 2)
     B.shingle_graph_destroy(h)
     return g, cfg, out
 
@@ -137,3 +148,31 @@ def test_fullsize_overlapping_clusters(run):
         row = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
         cons = oracle.row_constituents(row, cfg["s1"], int(A[j]), int(Bv[j]))
         assert clustered[cons].all()
+
+
+def test_fullsize_density(run):
+    """Eq. 6 at full size: the sampled clusters' density matches the oracle's
+    edge-by-edge count (fp64, same formula); all-cluster statistics are in
+    [0, 1] over exactly the clusters report_dense_subgraphs counts."""
+    g, cfg, out = run
+    mean, sd, nc = out["dens_s"]
+    members = np.flatnonzero(out["lab_s"] != np.arange(g.n))
+    keep = np.unique(out["lab_s"][members])
+    sub = np.union1d(members, keep)                    # vertices of the sampled clusters
+    # the oracle on the induced CSR of the sampled clusters (ids remapped)
+    remap = -np.ones(g.n, np.int64)
+    remap[sub] = np.arange(len(sub))
+    rp = [0]
+    cols = []
+    for u in sub:
+        row = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
+        row = remap[row[remap[row] >= 0]]
+        cols.append(np.sort(row))
+        rp.append(rp[-1] + len(row))
+    col = np.concatenate(cols).astype(np.int32)
+    lab = remap[out["lab_s"][sub]]
+    rm, rs, rn = oracle.cluster_density(np.asarray(rp, np.int64), col, lab, 2)
+    assert nc == rn == 30
+    assert abs(mean - rm) <= 1e-12 and abs(sd - rs) <= 1e-12
+    mean, sd, nc = out["dens20"]
+    assert nc == out["nc20"] and 0.0 < mean <= 1.0 and 0.0 <= sd <= 0.5

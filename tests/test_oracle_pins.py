@@ -433,3 +433,38 @@ def test_overlapping_inside_union_find_clusters():
     assert len(offs) > 1
     for i in range(len(offs) - 1):
         assert len(set(labels[verts[offs[i]:offs[i + 1]]].tolist())) == 1
+
+
+# ---------------------------------------------------------------- density (Eq. 6)
+def test_density_closed_forms():
+    """Cliques have density 1; a k-cycle has k / C(k, 2) = 2 / (k - 1); a
+    star on k vertices has (k - 1) / C(k, 2) = 2 / k; singletons are skipped."""
+    g = SG.cliques([5, 7, 9], n=30, seed=2)
+    lab = np.arange(g.n)
+    comp = _components(g)
+    for v in range(g.n):
+        lab[v] = comp[v]
+    mean, sd, nc = oracle.cluster_density(g.row_ptr, g.col, lab)
+    assert (mean, sd, nc) == (1.0, 0.0, 3)
+    # cycle 0-1-...-9 and a star centred at 10 with leaves 11..15, as one CSR
+    adj = {v: set() for v in range(16)}
+    for i in range(10):
+        adj[i].add((i + 1) % 10)
+        adj[(i + 1) % 10].add(i)
+    for leaf in range(11, 16):
+        adj[10].add(leaf)
+        adj[leaf].add(10)
+    rp = np.zeros(17, np.int64)
+    for v in range(16):
+        rp[v + 1] = rp[v] + len(adj[v])
+    col = np.concatenate([sorted(adj[v]) for v in range(16)]).astype(np.int32)
+    lab = np.array([0] * 10 + [10] * 6)
+    mean, sd, nc = oracle.cluster_density(rp, col, lab)
+    want = [2 / 9, 2 / 6]
+    assert nc == 2 and math.isclose(mean, np.mean(want)) and math.isclose(sd, np.std(want))
+    # splitting the cycle in halves: each half is a path of 5 (4 edges / 10)
+    lab2 = np.array([0] * 5 + [5] * 5 + [10] * 6)
+    mean, _, nc = oracle.cluster_density(rp, col, lab2, min_size=6)
+    assert nc == 1 and math.isclose(mean, 2 / 6)
+    mean, _, nc = oracle.cluster_density(rp, col, lab2)
+    assert nc == 3 and math.isclose(mean, (0.4 + 0.4 + 2 / 6) / 3)

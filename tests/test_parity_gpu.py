@@ -277,3 +277,28 @@ def test_overlapping_errors(B):
         G.run(2, 8, 1, 2, 8, 2)
         with pytest.raises(B.SGError):
             G.report_overlapping(2)          # bad mode
+
+
+# ---------------------------------------------------------------- density (Eq. 6)
+def test_density_tiny_and_cliques(B):
+    """Device intra-cluster edge counts vs the oracle on the tiny config's
+    reported clusters (both modes, min_size 2 and 20) and on planted cliques
+    (density exactly 1)."""
+    g = SG.make("tiny")
+    cfg = SG.CONFIGS["tiny"]
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        G.run(cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+        for mode in (0, 1):
+            labels, _ = G.report(mode)
+            for ms in (2, 20):
+                got = G.density(labels, ms)
+                want = oracle.cluster_density(g.row_ptr, g.col, labels, ms)
+                assert got[2] == want[2]
+                assert abs(got[0] - want[0]) <= 1e-12 and abs(got[1] - want[1]) <= 1e-12
+        with pytest.raises(B.SGError):
+            G.density(np.full(g.n, g.n, np.int32))      # label out of range
+    gc = SG.cliques([5, 8, 13], n=40, seed=6)
+    with B.ShingleGraph(gc.row_ptr, gc.col) as G:
+        G.run(2, 50, 1, 2, 50, 2)
+        labels, nc = G.report(0)
+        assert nc == 3 and G.density(labels) == (1.0, 0.0, 3)
