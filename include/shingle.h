@@ -173,6 +173,21 @@ SG_API sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t 
 SG_API sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_size,
                                     double *mean, double *stddev, int64_t *n_clusters);
 
+/* ------------------------------------------------------------------------ */
+/* sg_partition_agreement — the pair counts behind Eq. 2-5 (P:L1038-1060,  */
+/* AMB-15): over all unordered vertex pairs (i, j) of G,                    */
+/*   TP: same cluster in test and in benchmark;  FP: same in test only;     */
+/*   FN: same in benchmark only;                 TN: apart in both.         */
+/* PPV = TP/(TP+FP), NPV = TN/(TN+FN), SP = TN/(TN+FP), SE = TP/(TP+FN).    */
+/*   test_labels, bench_labels  host int32[n], values in [0, n) (borrowed). */
+/*   counts     receives {TP, FP, FN, TN} (exact 64-bit integers).          */
+/* Marginal histograms and a radix sort + run-length encode of the joint    */
+/* (test, benchmark) cells on the device.  Any state after create; world   */
+/* == 1.  Errors: SG_EINVAL (NULL, label out of range), SG_EOVERFLOW, ...   */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
+                                        const int32_t *bench_labels, int64_t counts[4]);
+
 /* Return the handle to state CREATED (CSR kept, results dropped) so the two */
 /* passes can be run again, e.g. by a benchmark.                             */
 SG_API sg_status shingle_graph_reset(sg_graph *g);

@@ -59,6 +59,7 @@ def lib() -> C.CDLL:
         "report_dense_subgraphs": (st, [vp, i32, i32, vp, vp]),
         "report_overlapping_clusters": (st, [vp, i32, i32, vp, vp, vp, vp]),
         "sg_cluster_density": (st, [vp, vp, i32, vp, vp, vp]),
+        "sg_partition_agreement": (st, [vp, vp, vp, vp]),
         "shingle_graph_reset": (st, [vp]),
         "shingle_graph_destroy": (None, [vp]),
         "sg_last_error": (C.c_char_p, [vp]),
@@ -161,6 +162,20 @@ def sg_cluster_density(h, labels, min_size: int = 2):
     _check(lib().sg_cluster_density(h, labels.ctypes.data, min_size, C.byref(mean), C.byref(sd),
                                     C.byref(nc)), h)
     return mean.value, sd.value, nc.value
+
+
+def sg_partition_agreement(h, test_labels, bench_labels) -> dict:
+    """Pair counts TP, FP, FN, TN and Eq. 2-5 (PPV, NPV, SP, SE)."""
+    t = np.ascontiguousarray(test_labels, np.int32)
+    b = np.ascontiguousarray(bench_labels, np.int32)
+    cnt = np.zeros(4, np.int64)
+    _check(lib().sg_partition_agreement(h, t.ctypes.data, b.ctypes.data, cnt.ctypes.data), h)
+    tp, fp, fn, tn = (int(x) for x in cnt)
+
+    def ratio(a, b):
+        return a / b if b else float("nan")
+    return dict(TP=tp, FP=fp, FN=fn, TN=tn, PPV=ratio(tp, tp + fp), NPV=ratio(tn, tn + fn),
+                SP=ratio(tn, tn + fp), SE=ratio(tp, tp + fn))
 
 
 def shingle_graph_reset(h):
@@ -286,6 +301,9 @@ class ShingleGraph:
 
     def report(self, mode=0, min_size=1):
         return report_dense_subgraphs(self.h, mode, min_size, self.n)
+
+    def agreement(self, test_labels, bench_labels):
+        return sg_partition_agreement(self.h, test_labels, bench_labels)
 
     def density(self, labels, min_size=2):
         return sg_cluster_density(self.h, labels, min_size)

@@ -1616,4 +1616,44 @@ sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_siz
   });
 }
 
+sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
+                                 const int32_t *bench_labels, int64_t counts[4]) {
+  return guarded(g, [&] {
+    if (!test_labels || !bench_labels || !counts) fail(g, SG_EINVAL, "NULL argument");
+    if (g->world > 1) require_single(g, "sg_partition_agreement");
+    const int64_t n = g->n;
+    if (n > INT32_MAX) fail(g, SG_EOVERFLOW, "n > 2^31");
+    for (int64_t v = 0; v < n; ++v)
+      if (test_labels[v] < 0 || test_labels[v] >= n || bench_labels[v] < 0 || bench_labels[v] >= n)
+        fail(g, SG_EINVAL, "labels must lie in [0, n)");
+    const size_t tb = agreement_temp_bytes(n);
+    DBuf dt, db, ct, cb, cj, k1, k2, temp, runs, out;
+    dalloc(g, dt, (size_t)n * 4);
+    dalloc(g, db, (size_t)n * 4);
+    dalloc(g, ct, (size_t)n * 4);
+    dalloc(g, cb, (size_t)n * 4);
+    dalloc(g, cj, (size_t)n * 4);
+    dalloc(g, k1, (size_t)n * 8);
+    dalloc(g, k2, (size_t)n * 8);
+    dalloc(g, temp, tb);
+    dalloc(g, runs, 8);
+    dalloc(g, out, 24);
+    CK(cudaMemcpyAsync(dt.p, test_labels, (size_t)n * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(cudaMemcpyAsync(db.p, bench_labels, (size_t)n * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(agreement_device(ptr<int32_t>(dt), ptr<int32_t>(db), n, ptr<uint32_t>(ct),
+                        ptr<uint32_t>(cb), ptr<uint32_t>(cj), ptr<uint64_t>(k1), ptr<uint64_t>(k2),
+                        temp.p, temp.bytes, ptr<int64_t>(runs), ptr<unsigned long long>(out),
+                        g->num_sms, g->stream));
+    unsigned long long h[3] = {0, 0, 0};
+    CK(cudaMemcpyAsync(h, out.p, 24, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    for (DBuf *b : {&dt, &db, &ct, &cb, &cj, &k1, &k2, &temp, &runs, &out}) dfree(g, *b);
+    const unsigned long long all = (unsigned long long)n * (unsigned long long)(n > 0 ? n - 1 : 0) / 2;
+    counts[0] = (int64_t)h[0];                          // TP: together in both
+    counts[1] = (int64_t)(h[1] - h[0]);                 // FP: together in test only
+    counts[2] = (int64_t)(h[2] - h[0]);                 // FN: together in benchmark only
+    counts[3] = (int64_t)(all - h[1] - h[2] + h[0]);    // TN: apart in both
+  });
+}
+
 }  // extern "C"

@@ -166,6 +166,15 @@ cudaError_t density_device(const int64_t *row_ptr, const uint32_t *col, int64_t 
                            const int32_t *labels, unsigned long long *e2, uint32_t *size,
                            int num_sms, cudaStream_t st);
 
+// Partition agreement (Eq. 2-5): t, b device int32[n] in [0, n); ct, cb, cj
+// uint32[n], key, key2 uint64[n] scratch; d_out3 <- {sum C(n_tb,2),
+// sum C(n_t,2), sum C(n_b,2)}.
+size_t agreement_temp_bytes(int64_t n);
+cudaError_t agreement_device(const int32_t *t, const int32_t *b, int64_t n, uint32_t *ct,
+                             uint32_t *cb, uint32_t *cj, uint64_t *key, uint64_t *key2, void *temp,
+                             size_t temp_bytes, int64_t *d_runs, unsigned long long *d_out3,
+                             int num_sms, cudaStream_t st);
+
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);

@@ -134,7 +134,7 @@ def homology_graph(n, n_isolated=0, m_target=None, seed=0,
                    n_cliques=0, clique_lo=10, clique_hi=60,
                    cc_exp=2.0, cc_lo=2, cc_max=10707,
                    fam_exp=2.0, fam_lo=4, fam_hi=600, dens_lo=0.3, dens_hi=0.9,
-                   linkers=4.0, n_hubs=0, hub_lo=10001, hub_hi=20000):
+                   linkers=4.0, n_hubs=0, hub_lo=10001, hub_hi=20000, return_families=False):
     rng = np.random.default_rng(seed)
     perm = rng.permutation(n).astype(np.int64)          # slot -> vertex id
     ea, eb = [], []
@@ -210,7 +210,22 @@ def homology_graph(n, n_isolated=0, m_target=None, seed=0,
     lo = perm[codes // n]
     hi = perm[codes % n]
     row_ptr, col = _csr_from_pairs(n, lo, hi)
-    return row_ptr, col
+    if not return_families:
+        return row_ptr, col
+    # planted partition (the "benchmark" of Eq. 2-5): cliques and families;
+    # isolated vertices alone.  Label = smallest vertex id of the family.
+    fam_of_slot = np.arange(n, dtype=np.int64)
+    s0 = n_isolated
+    for k in (ks if n_cliques else []):
+        fam_of_slot[s0:s0 + int(k)] = s0
+        s0 += int(k)
+    for base, size in zip(fam_base, fam_sizes):
+        fam_of_slot[base:base + size] = base
+    fam_min = np.full(n, n, np.int64)
+    np.minimum.at(fam_min, fam_of_slot, perm)
+    fam = np.empty(n, np.int32)
+    fam[perm] = fam_min[fam_of_slot]
+    return row_ptr, col, fam
 
 
 def _codes(n, a, b):

@@ -468,3 +468,24 @@ def test_density_closed_forms():
     assert nc == 1 and math.isclose(mean, 2 / 6)
     mean, _, nc = oracle.cluster_density(rp, col, lab2)
     assert nc == 3 and math.isclose(mean, (0.4 + 0.4 + 2 / 6) / 3)
+
+
+# ---------------------------------------------------------------- Eq. 2-5 pair counts
+def test_agreement_closed_forms():
+    """Identical partitions: FP = FN = 0, PPV = SE = 1; all-singletons test
+    vs one block of n: TP = 0, FN = C(n, 2); counts always sum to C(n, 2);
+    a hand-counted 5-vertex case; symmetric under swapping the roles (FP <-> FN)."""
+    rng = np.random.default_rng(3)
+    lab = rng.integers(0, 7, 60)
+    r = oracle.partition_agreement(lab, lab)
+    assert r["FP"] == r["FN"] == 0 and r["PPV"] == r["SE"] == 1.0
+    n = 40
+    r = oracle.partition_agreement(np.arange(n), np.zeros(n, int))
+    assert r["TP"] == 0 and r["FN"] == n * (n - 1) // 2 and r["FP"] == r["TN"] == 0
+    # test {0,1,2}{3,4}; benchmark {0,1}{2,3,4}: pairs 01 TP; 02,12 FP; 23,24 FN; 34 TP; rest TN (4)
+    r = oracle.partition_agreement([0, 0, 0, 3, 3], [0, 0, 2, 2, 2])
+    assert (r["TP"], r["FP"], r["FN"], r["TN"]) == (2, 2, 2, 4)
+    a, b = rng.integers(0, 5, 50), rng.integers(0, 9, 50)
+    r, q = oracle.partition_agreement(a, b), oracle.partition_agreement(b, a)
+    assert (r["TP"], r["FP"], r["FN"], r["TN"]) == (q["TP"], q["FN"], q["FP"], q["TN"])
+    assert r["TP"] + r["FP"] + r["FN"] + r["TN"] == 50 * 49 // 2

@@ -302,3 +302,35 @@ def test_density_tiny_and_cliques(B):
         G.run(2, 50, 1, 2, 50, 2)
         labels, nc = G.report(0)
         assert nc == 3 and G.density(labels) == (1.0, 0.0, 3)
+
+
+# ---------------------------------------------------------------- Eq. 2-5 pair counts
+def test_agreement_vs_planted_families(B):
+    """TP/FP/FN/TN of the reported clusters against the generator's planted
+    families (the benchmark partition of Eq. 2-5), both report modes, and of
+    mode 0 against mode 1 on the tiny config: exact integers vs the oracle's
+    pair-by-pair count."""
+    row_ptr, col, fam = SG.homology_graph(n=3000, n_isolated=300, m_target=40000, seed=41,
+                                          n_cliques=12, clique_lo=6, clique_hi=30, cc_max=600,
+                                          fam_hi=200, return_families=True)
+    g = SG.Graph(row_ptr, col)
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        G.run(2, 60, 141, 2, 60, 241)
+        for mode in (0, 1):
+            labels, _ = G.report(mode)
+            got = G.agreement(labels, fam)
+            want = oracle.partition_agreement(labels, fam)
+            assert {k: got[k] for k in ("TP", "FP", "FN", "TN")} == \
+                   {k: want[k] for k in ("TP", "FP", "FN", "TN")}
+            assert got["TP"] > 0
+        with pytest.raises(B.SGError):
+            G.agreement(np.full(g.n, -1, np.int32), fam)
+    t = SG.make("tiny")
+    cfg = SG.CONFIGS["tiny"]
+    with B.ShingleGraph(t.row_ptr, t.col) as G:
+        G.run(cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+        l0, _ = G.report(0)
+        l1, _ = G.report(1)
+        got = G.agreement(l0, l1)
+        want = oracle.partition_agreement(l0, l1)
+        assert [got[k] for k in ("TP", "FP", "FN", "TN")] == [want[k] for k in ("TP", "FP", "FN", "TN")]
