@@ -188,6 +188,20 @@ SG_API sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t 
 SG_API sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
                                         const int32_t *bench_labels, int64_t counts[4]);
 
+/* ------------------------------------------------------------------------ */
+/* sg_connected_components — the connected components of G, the            */
+/* decomposition pClust applies before shingling: no dense     */
+/* subgraph spans two components, so each can be shingled on its own.     */
+/*   labels        host int32[n], caller-allocated; labels[v] = smallest    */
+/*                 vertex of v's component (isolated vertices: v).          */
+/*   n_components  receives the number of components (may be NULL).        */
+/* Lock-free union-find over n on the device (one warp per CSR row, each    */
+/* stored entry (u, v) is an undirected edge).  Any state after create;   */
+/* world == 1.                                                              */
+/* Errors: SG_EINVAL (NULL labels), SG_ESTATE, SG_ENOMEM, SG_ECUDA.         */
+/* ------------------------------------------------------------------------ */
+SG_API sg_status sg_connected_components(sg_graph *g, int32_t *labels, int64_t *n_components);
+
 /* Return the handle to state CREATED (CSR kept, results dropped) so the two */
 /* passes can be run again, e.g. by a benchmark.                             */
 SG_API sg_status shingle_graph_reset(sg_graph *g);

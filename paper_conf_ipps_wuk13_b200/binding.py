@@ -60,6 +60,7 @@ def lib() -> C.CDLL:
         "report_overlapping_clusters": (st, [vp, i32, i32, vp, vp, vp, vp]),
         "sg_cluster_density": (st, [vp, vp, i32, vp, vp, vp]),
         "sg_partition_agreement": (st, [vp, vp, vp, vp]),
+        "sg_connected_components": (st, [vp, vp, vp]),
         "shingle_graph_reset": (st, [vp]),
         "shingle_graph_destroy": (None, [vp]),
         "sg_last_error": (C.c_char_p, [vp]),
@@ -176,6 +177,16 @@ def sg_partition_agreement(h, test_labels, bench_labels) -> dict:
         return a / b if b else float("nan")
     return dict(TP=tp, FP=fp, FN=fn, TN=tn, PPV=ratio(tp, tp + fp), NPV=ratio(tn, tn + fn),
                 SP=ratio(tn, tn + fp), SE=ratio(tp, tp + fn))
+
+
+def sg_connected_components(h, n: Optional[int] = None):
+    """Connected components of G: (labels int32[n] = smallest vertex, count)."""
+    if n is None:
+        n = sg_get_counts(h)["n"]
+    labels = np.zeros(n, np.int32)
+    nc = C.c_int64()
+    _check(lib().sg_connected_components(h, labels.ctypes.data, C.byref(nc)), h)
+    return labels, nc.value
 
 
 def shingle_graph_reset(h):
@@ -301,6 +312,9 @@ class ShingleGraph:
 
     def report(self, mode=0, min_size=1):
         return report_dense_subgraphs(self.h, mode, min_size, self.n)
+
+    def components(self):
+        return sg_connected_components(self.h, self.n)
 
     def agreement(self, test_labels, bench_labels):
         return sg_partition_agreement(self.h, test_labels, bench_labels)

@@ -1656,4 +1656,26 @@ sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
   });
 }
 
+sg_status sg_connected_components(sg_graph *g, int32_t *labels, int64_t *n_components) {
+  return guarded(g, [&] {
+    if (!labels) fail(g, SG_EINVAL, "labels is NULL");
+    if (g->world > 1) require_single(g, "sg_connected_components");
+    const int64_t n = g->n;
+    DBuf parent, dl;
+    dalloc(g, parent, (size_t)n * 4);
+    dalloc(g, dl, (size_t)n * 4);
+    CK(components_device(ptr<int64_t>(g->row_ptr), ptr<uint32_t>(g->col), n,
+                         ptr<uint32_t>(parent), ptr<int32_t>(dl), g->num_sms, g->stream));
+    if (n) CK(cudaMemcpyAsync(labels, dl.p, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    dfree(g, parent);
+    dfree(g, dl);
+    if (n_components) {
+      int64_t c = 0;
+      for (int64_t v = 0; v < n; ++v) c += labels[v] == (int32_t)v;
+      *n_components = c;
+    }
+  });
+}
+
 }  // extern "C"

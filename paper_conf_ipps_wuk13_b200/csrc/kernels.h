@@ -175,6 +175,11 @@ cudaError_t agreement_device(const int32_t *t, const int32_t *b, int64_t n, uint
                              size_t temp_bytes, int64_t *d_runs, unsigned long long *d_out3,
                              int num_sms, cudaStream_t st);
 
+// Connected components of G: parent uint32[n] scratch, labels device int32[n]
+// <- smallest vertex of the component.
+cudaError_t components_device(const int64_t *row_ptr, const uint32_t *col, int64_t n,
+                              uint32_t *parent, int32_t *labels, int num_sms, cudaStream_t st);
+
 // ---- getters (kernels_group.cu) --------------------------------------------
 cudaError_t popcount_words(const uint32_t *w, int64_t nwords, unsigned long long *d_out,
                            cudaStream_t st);

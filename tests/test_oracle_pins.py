@@ -489,3 +489,24 @@ def test_agreement_closed_forms():
     r, q = oracle.partition_agreement(a, b), oracle.partition_agreement(b, a)
     assert (r["TP"], r["FP"], r["FN"], r["TN"]) == (q["TP"], q["FN"], q["FP"], q["TN"])
     assert r["TP"] + r["FP"] + r["FN"] + r["TN"] == 50 * 49 // 2
+
+
+# ---------------------------------------------------------------- connected components
+def test_components_vs_bfs():
+    """scipy-based components = a plain BFS (this file's _components), on the
+    homology generator's graphs and on cliques; labels are the minimum vertex."""
+    for gseed in (1, 2):
+        g = SG.Graph(*SG.homology_graph(n=400, n_isolated=30, m_target=2500, seed=gseed,
+                                        n_cliques=3, clique_lo=6, clique_hi=12, cc_max=60,
+                                        fam_hi=40))
+        lab, k = oracle.connected_components(g.row_ptr, g.col)
+        comp = _components(g)
+        by = defaultdict(list)
+        for v in range(g.n):
+            by[comp[v]].append(v)
+        assert k == len(by)
+        for members in by.values():
+            assert set(lab[members].tolist()) == {min(members)}
+    # an asymmetric CSR (edge 0 -> 3 stored once) still joins 0 and 3
+    lab, k = oracle.connected_components(np.array([0, 1, 1, 1, 1]), np.array([3], np.int32))
+    assert lab.tolist() == [0, 1, 2, 0] and k == 3

@@ -334,3 +334,20 @@ def test_agreement_vs_planted_families(B):
         got = G.agreement(l0, l1)
         want = oracle.partition_agreement(l0, l1)
         assert [got[k] for k in ("TP", "FP", "FN", "TN")] == [want[k] for k in ("TP", "FP", "FN", "TN")]
+
+
+# ---------------------------------------------------------------- connected components
+@pytest.mark.parametrize("name", ["tiny", "small", "cliques"])
+def test_components(B, name):
+    if name == "tiny":
+        g = SG.make("tiny")
+    elif name == "small":
+        g = SG.Graph(*SG.homology_graph(n=30000, n_isolated=3000, m_target=300000, seed=51,
+                                        n_cliques=20, clique_lo=6, clique_hi=40, cc_max=3000,
+                                        fam_hi=300))
+    else:
+        g = SG.cliques([5, 8, 13, 40], n=100, seed=6)
+    with B.ShingleGraph(g.row_ptr, g.col) as G:
+        lab, k = G.components()
+    want, wk = oracle.connected_components(g.row_ptr, g.col)
+    assert k == wk and np.array_equal(lab, want)
