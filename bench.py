@@ -252,7 +252,7 @@ def bench_ours(args, rank, world, local_rank):
     # Phase III on the device, outside the metric: clusters of
     # >= 20 vertices (the size the paper evaluated)
     phase3 = None
-    if world == 1:
+    if world == 1 and not args.no_phase3:
         lab20, ncl = B.report_dense_subgraphs(h, 0, 20, g.n)
         phase3 = {"ms": round(B.sg_get_stage_ms(h).get("report", 0.0), 3), "clusters_ge20": int(ncl),
                   "mode": "constituents (AMB-9)", "timed_in_metric": False}
@@ -384,6 +384,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="gos2m")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-phase3", action="store_true", help="skip the untimed Phase III reports")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-nnz", type=int, default=1_500_000)
     ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
