@@ -127,7 +127,7 @@ SG_API sg_status group_by_shingle(sg_graph *g);
 /*              G_II pair, stage "report" of sg_get_stage_ms); with the flag:  */
 /*              the same union-find on the host (G_I, G_II copied back).       */
 /* Outside the timed two-pass hot path.  Requires state GROUPED2 and         */
-/* world == 1 (SG_ESTATE otherwise: gather G_II with sg_get_groups).         */
+/* world == 1 (SG_EINVAL otherwise: gather G_II with sg_get_groups).         */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, int32_t *labels,
                                  int64_t *n_clusters);
@@ -148,7 +148,8 @@ SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_s
 /*            each call recomputes on the device).                          */
 /* Union-find over S1', constituent emission, radix sort + unique on the    */
 /* device; the host splits the sorted list.  Untimed; state GROUPED2,       */
-/* world == 1.  Errors: SG_EINVAL (mode, NULL counts, caps too small),      */
+/* world == 1.  Errors: SG_EINVAL (mode, NULL counts, caps too small,       */
+/* world > 1),                                                               */
 /* SG_ESTATE, SG_ENOMEM, SG_ECUDA, SG_EOVERFLOW (> 2^31 constituents).      */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_size,
@@ -168,7 +169,7 @@ SG_API sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t 
 /* Intra-cluster edges are counted on the device (one warp per row, over   */
 /* the resident CSR; undirected edges are stored twice, AMB-11).  Any state */
 /* after create; world == 1.  Errors: SG_EINVAL (NULL labels, label out of  */
-/* range), SG_ESTATE, SG_ENOMEM, SG_ECUDA.                                   */
+/* range, world > 1), SG_ENOMEM, SG_ECUDA.                                  */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_size,
                                     double *mean, double *stddev, int64_t *n_clusters);
@@ -183,7 +184,8 @@ SG_API sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t 
 /*   counts     receives {TP, FP, FN, TN} (exact 64-bit integers).          */
 /* Marginal histograms and a radix sort + run-length encode of the joint    */
 /* (test, benchmark) cells on the device.  Any state after create; world   */
-/* == 1.  Errors: SG_EINVAL (NULL, label out of range), SG_EOVERFLOW, ...   */
+/* == 1.  Errors: SG_EINVAL (NULL, label out of range, world > 1),         */
+/* SG_EOVERFLOW, SG_ENOMEM, SG_ECUDA.                                      */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
                                         const int32_t *bench_labels, int64_t counts[4]);
@@ -198,7 +200,7 @@ SG_API sg_status sg_partition_agreement(sg_graph *g, const int32_t *test_labels,
 /* Lock-free union-find over n on the device (one warp per CSR row, each    */
 /* stored entry (u, v) is an undirected edge).  Any state after create;   */
 /* world == 1.                                                              */
-/* Errors: SG_EINVAL (NULL labels), SG_ESTATE, SG_ENOMEM, SG_ECUDA.         */
+/* Errors: SG_EINVAL (NULL labels, world > 1), SG_ENOMEM, SG_ECUDA.       */
 /* ------------------------------------------------------------------------ */
 SG_API sg_status sg_connected_components(sg_graph *g, int32_t *labels, int64_t *n_components);
 

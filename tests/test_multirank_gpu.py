@@ -196,3 +196,42 @@ def test_loopback_peer_failure_does_not_hang(B):
     assert not any(t.is_alive() for t in ts)
     B.sg_loopback_destroy(lb)
     assert errs[1] == B.SG_ESTATE and errs[0] == B.SG_ESTATE
+
+
+def test_loopback_single_rank_calls_refuse_world_gt_1(B):
+    """The report and quality calls are single-rank: with world > 1
+    they fail with SG_EINVAL on every rank instead of computing a partial answer."""
+    g = SG.make("tiny")
+    lb = B.sg_loopback_create(2)
+    codes = [[], []]
+
+    def body(r):
+        h = B.shingle_graph_create(g.row_ptr, g.col,
+                                   dist={"rank": r, "world": 2, "device": 0, "loopback": lb})
+        try:
+            B.shingle_pass(h, 2, 8, 1)
+            B.group_by_shingle(h)
+            B.shingle_pass(h, 2, 8, 2)
+            B.group_by_shingle(h)
+            lab = np.arange(g.n, dtype=np.int32)
+            for call in (lambda: B.report_dense_subgraphs(h, 0, 1, g.n),
+                         lambda: B.report_overlapping_clusters(h, 0),
+                         lambda: B.sg_cluster_density(h, lab),
+                         lambda: B.sg_partition_agreement(h, lab, lab),
+                         lambda: B.sg_connected_components(h, g.n)):
+                try:
+                    call()
+                    codes[r].append(0)
+                except B.SGError as e:
+                    codes[r].append(e.status)
+        finally:
+            B.shingle_graph_destroy(h)
+
+    ts = [threading.Thread(target=body, args=(r,)) for r in range(2)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(120)
+    assert not any(t.is_alive() for t in ts)
+    B.sg_loopback_destroy(lb)
+    assert codes == [[B.SG_EINVAL] * 5, [B.SG_EINVAL] * 5]
