@@ -100,6 +100,16 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
     e = cudaMallocAsync(&p, bytes, g->stream);
   }
   if (e != cudaSuccess) {
+    // the pool's free blocks may be too fragmented for one large request
+    // (e.g. after a step with another (s, c)): return them to the device and
+    // map the request afresh
+    cudaGetLastError();
+    cudaStreamSynchronize(g->stream);
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, g->device) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
+    e = cudaMallocAsync(&p, bytes, g->stream);
+  }
+  if (e != cudaSuccess) {
     cudaGetLastError();
     size_t fr = 0, tot = 0;
     cudaMemGetInfo(&fr, &tot);
