@@ -257,7 +257,7 @@ def bench_ours(args, rank, world, local_rank):
         phase3 = {"ms": round(B.sg_get_stage_ms(h).get("report", 0.0), 3), "clusters_ge20": int(ncl),
                   "mode": "constituents (AMB-9)", "timed_in_metric": False}
         # approach 1 (overlapping clusters), host-timed: both calls of
-        # the two-call pattern (sizes, then fill), each recomputing on the device
+        # the two-call pattern (sizes, then fill from the kept result)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         ooffs, _ = B.report_overlapping_clusters(h, 0, 20)

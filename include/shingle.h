@@ -145,7 +145,8 @@ SG_API sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_s
 /*            verts[offs[i], offs[i+1]), vertices ascending; clusters in     */
 /*            order of their smallest S1' index.  Caller-allocated; caps =   */
 /*            {C+1, V}.  Both NULL: only counts <- {C, V} (two-call pattern; */
-/*            each call recomputes on the device).                          */
+/*            the sizing call's result is kept on the host for the next     */
+/*            filling call with the same mode and min_size, then released). */
 /* Union-find over S1', constituent emission, radix sort + unique on the    */
 /* device; the host splits the sorted list.  Untimed; state GROUPED2,       */
 /* world == 1.  Errors: SG_EINVAL (mode, NULL counts, caps too small,       */

@@ -1178,6 +1178,7 @@ sg_status shingle_graph_reset(sg_graph *g) {
     }
     sync(g);
     g->e2_global = -1;
+    g->ov_valid = false;
     g->launch_base = g_launches.load();
     g->state = kCreated;
   });
@@ -1498,13 +1499,7 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
   });
 }
 
-sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_size, int64_t *offs,
-                                      uint32_t *verts, const int64_t caps[2], int64_t counts[2]) {
-  return guarded(g, [&] {
-    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
-    if (!counts) fail(g, SG_EINVAL, "counts is NULL");
-    if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
-    if (g->world > 1) require_single(g, "report_overlapping_clusters");
+static void overlap_compute(sg_graph *g, int32_t mode, int32_t min_size) {
     PassOut &P1 = g->pass[0];
     PassOut &P2 = g->pass[1];
     ReportArgs a;
@@ -1557,28 +1552,40 @@ sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_siz
     if (nu && u[(size_t)nu - 1] == ~0ull) --nu;         // rows shorter than s1 (none in practice)
     // split the sorted (root, vertex) list into clusters; drop the small ones
     const int64_t thr = std::max<int32_t>(1, min_size);
-    int64_t nc = 0, nv = 0;
+    g->ov_offs.assign(1, 0);
+    g->ov_verts.clear();
     for (int64_t i = 0; i < nu;) {
       int64_t e = i + 1;
       while (e < nu && (u[(size_t)e] >> 32) == (u[(size_t)i] >> 32)) ++e;
       if (e - i >= thr) {
-        if (offs || verts) {
-          if (!caps || caps[0] < nc + 2 || caps[1] < nv + (e - i)) fail(g, SG_EINVAL, "buffers too small");
-          if (offs) {
-            offs[nc] = nv;
-            offs[nc + 1] = nv + (e - i);
-          }
-          if (verts)
-            for (int64_t x = i; x < e; ++x) verts[nv + (x - i)] = (uint32_t)u[(size_t)x];
-        }
-        ++nc;
-        nv += e - i;
+        for (int64_t x = i; x < e; ++x) g->ov_verts.push_back((uint32_t)u[(size_t)x]);
+        g->ov_offs.push_back((int64_t)g->ov_verts.size());
       }
       i = e;
     }
-    if (offs && nc == 0) {
-      if (!caps || caps[0] < 1) fail(g, SG_EINVAL, "buffers too small");
-      offs[0] = 0;
+}
+
+sg_status report_overlapping_clusters(sg_graph *g, int32_t mode, int32_t min_size, int64_t *offs,
+                                      uint32_t *verts, const int64_t caps[2], int64_t counts[2]) {
+  return guarded(g, [&] {
+    if (mode != 0 && mode != 1) fail(g, SG_EINVAL, "mode must be 0 or 1");
+    if (!counts) fail(g, SG_EINVAL, "counts is NULL");
+    if (g->state != kGrouped2) fail(g, SG_ESTATE, "report needs both passes grouped");
+    if (g->world > 1) require_single(g, "report_overlapping_clusters");
+    if (!(g->ov_valid && g->ov_mode == mode && g->ov_min == min_size)) {
+      overlap_compute(g, mode, min_size);
+      g->ov_valid = true;
+      g->ov_mode = mode;
+      g->ov_min = min_size;
+    }
+    const int64_t nc = (int64_t)g->ov_offs.size() - 1, nv = (int64_t)g->ov_verts.size();
+    if (offs || verts) {
+      if (!caps || caps[0] < nc + 1 || caps[1] < nv) fail(g, SG_EINVAL, "buffers too small");
+      if (offs) std::copy(g->ov_offs.begin(), g->ov_offs.end(), offs);
+      if (verts) std::copy(g->ov_verts.begin(), g->ov_verts.end(), verts);
+      g->ov_valid = false;                              // filled: release the host copy
+      std::vector<int64_t>().swap(g->ov_offs);
+      std::vector<uint32_t>().swap(g->ov_verts);
     }
     counts[0] = nc;
     counts[1] = nv;

@@ -160,6 +160,13 @@ struct sg_graph {
   int64_t pairs_global[2] = {0, 0};
   int64_t e2_global = -1;       // pass-II entries (sum of |L| over S1'), lazily
   long long launch_base = 0;    // g_launches at create / reset
+  // report_overlapping_clusters two-call pattern: the sizing call keeps its
+  // result here for the filling call (same mode / min_size); cleared by it
+  // and by reset
+  bool ov_valid = false;
+  int32_t ov_mode = 0, ov_min = 0;
+  std::vector<int64_t> ov_offs;
+  std::vector<uint32_t> ov_verts;
   // stage timing: event pairs per stage (a stage may span several chunks)
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_next = 0;
