@@ -1554,6 +1554,7 @@ static void overlap_compute(sg_graph *g, int32_t mode, int32_t min_size) {
     const int64_t thr = std::max<int32_t>(1, min_size);
     g->ov_offs.assign(1, 0);
     g->ov_verts.clear();
+    g->ov_verts.reserve((size_t)nu);
     for (int64_t i = 0; i < nu;) {
       int64_t e = i + 1;
       while (e < nu && (u[(size_t)e] >> 32) == (u[(size_t)i] >> 32)) ++e;
