@@ -472,3 +472,270 @@ int32_t or_report(const or_result *R, int32_t mode, int32_t min_size, int32_t *l
     free(pc); free(cv); free(pv); free(first); free(size);
     return 0;
 }
+
+/* ---------------------------------------------------------------------- */
+/* Trial-outer streaming run of the same method, for graphs whose full     */
+/* outputs do not fit in host memory (the 2M and 640M configurations).     */
+/* The loop order of P:L445-460 (vertex-outer) versus trial-outer does not  */
+/* change any output, and grouping is per trial (AMB-5), so    */
+/* trial j of G_I depends only on column j of the pass-I matrix.  Pass I   */
+/* and G_I are computed one trial at a time for all c1 trials; the S1'     */
+/* nodes of trial j (groups with |L| >= s2) get their dense    */
+/* index k in canonical (trial, key) order and their pass-II shingles for  */
+/* the requested pass-II trials only (pass II "the same series of steps",  */
+/* P:L461-462); G_II is formed for those trials.  Kept: the pass-I columns */
+/* and G_I trials listed in keep1, the pass-II columns and G_II trials     */
+/* listed in keep2, the S1' map, counts, and per-trial digests of every    */
+/* pass-I column and G_I trial.                                            */
+/*                                                                          */
+/* Digest (test infrastructure, order- and position-sensitive): a column   */
+/* x_0..x_{N-1} digests to sum_i mix64(x_i + mix64(i)) mod 2^64; a grouped */
+/* trial with group ids id_g and members m_p (head bit h_p = 1 at the first */
+/* member of a group) to sum_g mix64(id_g + mix64(2g))                     */
+/*                     + sum_p mix64((m_p | h_p << 32) + mix64(2p + 1)).   */
+/* ---------------------------------------------------------------------- */
+static uint64_t dig_col_term(uint64_t x, uint64_t i) { return or_mix64(x + or_mix64(i)); }
+static uint64_t dig_gid_term(uint64_t id, uint64_t g) { return or_mix64(id + or_mix64(2 * g)); }
+static uint64_t dig_mem_term(uint32_t m, int head, uint64_t p)
+{
+    return or_mix64(((uint64_t)m | ((uint64_t)(head ? 1 : 0) << 32)) + or_mix64(2 * p + 1));
+}
+
+/* The within-trial id of one row for trial j: insertion top-s + id. */
+static uint64_t row_trial_id(const uint32_t *row, int64_t deg, int32_t s, uint64_t seed, int32_t j,
+                             uint32_t A, uint32_t B)
+{
+    uint32_t mins[16], argv[16];
+    top_s_insertion(row, deg, s, A, B, mins, argv);
+    return or_shingle_id(s, seed, j, mins);
+}
+
+typedef struct {
+    int64_t n, cap;
+    void *p;
+    size_t esz;
+} or_vec;
+
+static int vec_push(or_vec *v, const void *x)
+{
+    if (v->n == v->cap) {
+        int64_t nc = v->cap ? v->cap * 2 : 1024;
+        void *q = realloc(v->p, (size_t)nc * v->esz);
+        if (!q) return 1;
+        v->p = q;
+        v->cap = nc;
+    }
+    memcpy((char *)v->p + (size_t)v->n * v->esz, x, v->esz);
+    v->n++;
+    return 0;
+}
+
+typedef struct {
+    int32_t status;
+    int32_t c1, c2, nkeep1, nkeep2;
+    int64_t n_e, groups1, pairs1, n_s1p, e2;
+    uint32_t *rows1;          /* [n_e] */
+    uint64_t *dig_M1;         /* [c1] */
+    uint64_t *dig_G1;         /* [c1] */
+    uint64_t *M1k;            /* [n_e x nkeep1] columns keep1[] of the pass-I matrix */
+    or_groups G1k;            /* G_I restricted to trials keep1[] (c = nkeep1) */
+    int64_t *s1p_group;       /* [n_s1p] global G_I group index of S1' node k */
+    uint64_t *M2k;            /* [n_s1p x nkeep2] columns keep2[] of the pass-II matrix */
+    or_groups G2k;            /* G_II restricted to trials keep2[] */
+    uint64_t *dig_G2k;        /* [nkeep2] */
+} or_stream;
+
+static int in_list(const int32_t *l, int32_t n, int32_t x)
+{
+    for (int32_t i = 0; i < n; i++)
+        if (l[i] == x) return i;
+    return -1;
+}
+
+void or_stream_free(or_stream *S);
+
+or_stream *or_shingling_stream(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col,
+                               int32_t s1, int32_t c1, uint64_t seed1,
+                               int32_t s2, int32_t c2, uint64_t seed2,
+                               const int32_t *keep1, int32_t nkeep1,
+                               const int32_t *keep2, int32_t nkeep2)
+{
+    or_stream *S = (or_stream *)calloc(1, sizeof(or_stream));
+    if (!S) return NULL;
+    S->c1 = c1; S->c2 = c2; S->nkeep1 = nkeep1; S->nkeep2 = nkeep2;
+    if (s1 < 1 || s1 > 16 || s2 < 1 || s2 > 16 || c1 < 1 || c2 < 1 || nkeep1 < 0 || nkeep2 < 0 ||
+        or_validate(n, nnz, row_ptr, col)) {
+        S->status = 1;
+        return S;
+    }
+    uint32_t *A1 = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)c1);
+    uint32_t *B1 = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)c1);
+    uint32_t *A2 = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)c2);
+    uint32_t *B2 = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)c2);
+    or_hash_params(seed1, c1, A1, B1);
+    or_hash_params(seed2, c2, A2, B2);
+
+    /* pass-I rows: vertices with >= s1 links */
+    int64_t n_e = 0;
+    for (int64_t u = 0; u < n; u++)
+        if (row_ptr[u + 1] - row_ptr[u] >= s1) n_e++;
+    S->n_e = n_e;
+    S->rows1 = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(n_e > 0 ? n_e : 1));
+    for (int64_t u = 0, r = 0; u < n; u++)
+        if (row_ptr[u + 1] - row_ptr[u] >= s1) S->rows1[r++] = (uint32_t)u;
+    S->dig_M1 = (uint64_t *)calloc((size_t)c1, sizeof(uint64_t));
+    S->dig_G1 = (uint64_t *)calloc((size_t)c1, sizeof(uint64_t));
+    S->M1k = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)(n_e * nkeep1 > 0 ? n_e * nkeep1 : 1));
+    or_pair *pairs = (or_pair *)malloc((size_t)(n_e > 0 ? n_e : 1) * sizeof(or_pair));
+    or_pair *tmp = (or_pair *)malloc((size_t)(n_e > 0 ? n_e : 1) * sizeof(or_pair));
+    /* kept G_I trials (grown as they are cut) */
+    or_vec g1ids = {0, 0, NULL, sizeof(uint64_t)}, g1offs = {0, 0, NULL, sizeof(int64_t)};
+    or_vec g1mem = {0, 0, NULL, sizeof(uint32_t)};
+    S->G1k.c = nkeep1;
+    S->G1k.trial_goffs = (int64_t *)calloc((size_t)nkeep1 + 1, sizeof(int64_t));
+    /* S1' map and the kept pass-II columns */
+    or_vec s1p = {0, 0, NULL, sizeof(int64_t)};
+    or_vec m2 = {0, 0, NULL, sizeof(uint64_t) * (size_t)(nkeep2 > 0 ? nkeep2 : 1)};
+    uint64_t *m2row = (uint64_t *)calloc((size_t)(nkeep2 > 0 ? nkeep2 : 1), sizeof(uint64_t));
+    if (!A1 || !B1 || !A2 || !B2 || !S->rows1 || !S->dig_M1 || !S->dig_G1 || !S->M1k || !pairs ||
+        !tmp || !S->G1k.trial_goffs || !m2row) {
+        S->status = 2;
+        goto done;
+    }
+    int64_t g_glob = 0;    /* global G_I group index */
+    for (int32_t j = 0; j < c1; j++) {
+        const int32_t kj = in_list(keep1, nkeep1, j);
+        uint64_t dm = 0;
+        for (int64_t r = 0; r < n_e; r++) {                   /* emission order */
+            const uint32_t u = S->rows1[r];
+            const uint64_t id = row_trial_id((const uint32_t *)(col + row_ptr[u]),
+                                             row_ptr[u + 1] - row_ptr[u], s1, seed1, j, A1[j], B1[j]);
+            dm += dig_col_term(id, (uint64_t)r);
+            if (kj >= 0) S->M1k[r * nkeep1 + kj] = id;
+            pairs[r].id = id;
+            pairs[r].key = or_mix64(id);
+            pairs[r].member = u;
+        }
+        S->dig_M1[j] = dm;
+        merge_sort_by_key(pairs, tmp, 0, n_e);                  /* per-trial sorting (AMB-5) */
+        if (kj >= 0) S->G1k.trial_goffs[kj] = g1ids.n;           /* keep1 is given ascending */
+        uint64_t dg = 0;
+        int64_t gl = -1;       /* local group index within trial j */
+        for (int64_t r = 0; r < n_e;) {
+            int64_t e = r + 1;
+            while (e < n_e && pairs[e].key == pairs[r].key) e++;
+            gl++;
+            dg += dig_gid_term(pairs[r].id, (uint64_t)gl);
+            for (int64_t x = r; x < e; x++) dg += dig_mem_term(pairs[x].member, x == r, (uint64_t)x);
+            if (kj >= 0) {
+                int64_t off = g1mem.n;
+                if (vec_push(&g1ids, &pairs[r].id) || vec_push(&g1offs, &off)) { S->status = 2; goto done; }
+                for (int64_t x = r; x < e; x++)
+                    if (vec_push(&g1mem, &pairs[x].member)) { S->status = 2; goto done; }
+            }
+            const int64_t len = e - r;
+            if (len >= s2) {                                      /* S1' */
+                /* L(s): the generators, ascending (stable sort of ascending rows) */
+                uint32_t *L = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)len);
+                if (!L) { S->status = 2; goto done; }
+                for (int64_t x = r; x < e; x++) L[x - r] = pairs[x].member;
+                for (int32_t t2 = 0; t2 < nkeep2; t2++) {
+                    const int32_t t = keep2[t2];
+                    m2row[t2] = row_trial_id(L, len, s2, seed2, t, A2[t], B2[t]);
+                }
+                free(L);
+                if (vec_push(&s1p, &g_glob) || (nkeep2 > 0 && vec_push(&m2, m2row))) { S->status = 2; goto done; }
+                S->e2 += len;
+            }
+            g_glob++;
+            r = e;
+        }
+        S->dig_G1[j] = dg;
+        S->groups1 += gl + 1;
+        S->pairs1 += n_e;
+    }
+    S->G1k.trial_goffs[nkeep1] = g1ids.n;
+    S->G1k.ngroups = g1ids.n;
+    S->G1k.npairs = g1mem.n;
+    {
+        int64_t endoff = g1mem.n;
+        if (vec_push(&g1offs, &endoff)) { S->status = 2; goto done; }
+    }
+    S->G1k.ids = (uint64_t *)g1ids.p;
+    S->G1k.offs = (int64_t *)g1offs.p;
+    S->G1k.members = (uint32_t *)g1mem.p;
+    g1ids.p = g1offs.p = g1mem.p = NULL;
+    S->n_s1p = s1p.n;
+    S->s1p_group = (int64_t *)s1p.p;
+    s1p.p = NULL;
+    S->M2k = (uint64_t *)m2.p;
+    m2.p = NULL;
+    /* G_II for the kept pass-II trials: the same grouping (member = k) */
+    {
+        const int64_t nk = S->n_s1p;
+        uint64_t *col2 = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)(nk * (nkeep2 > 0 ? nkeep2 : 1) + 1));
+        uint32_t *kk = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(nk > 0 ? nk : 1));
+        S->dig_G2k = (uint64_t *)calloc((size_t)(nkeep2 > 0 ? nkeep2 : 1), sizeof(uint64_t));
+        if (!col2 || !kk || !S->dig_G2k) { free(col2); free(kk); S->status = 2; goto done; }
+        for (int64_t k = 0; k < nk; k++) kk[k] = (uint32_t)k;
+        /* group_pass wants the [rows x c] matrix: M2k already is [nk x nkeep2] */
+        if (nkeep2 > 0 && group_pass(nk, nkeep2, S->M2k, kk, &S->G2k)) {
+            free(col2); free(kk); S->status = 2; goto done;
+        }
+        if (nkeep2 == 0) {
+            S->G2k.trial_goffs = (int64_t *)calloc(1, sizeof(int64_t));
+            S->G2k.offs = (int64_t *)calloc(1, sizeof(int64_t));
+        }
+        for (int32_t t2 = 0; t2 < nkeep2; t2++) {
+            uint64_t d = 0;
+            const int64_t g0 = S->G2k.trial_goffs[t2], g1 = S->G2k.trial_goffs[t2 + 1];
+            const int64_t p0 = S->G2k.offs[g0];
+            for (int64_t g = g0; g < g1; g++) {
+                d += dig_gid_term(S->G2k.ids[g], (uint64_t)(g - g0));
+                for (int64_t p = S->G2k.offs[g]; p < S->G2k.offs[g + 1]; p++)
+                    d += dig_mem_term(S->G2k.members[p], p == S->G2k.offs[g], (uint64_t)(p - p0));
+            }
+            S->dig_G2k[t2] = d;
+        }
+        free(col2);
+        free(kk);
+    }
+    S->status = 0;
+done:
+    free(A1); free(B1); free(A2); free(B2);
+    free(pairs); free(tmp); free(m2row);
+    free(g1ids.p); free(g1offs.p); free(g1mem.p); free(s1p.p); free(m2.p);
+    return S;
+}
+
+void or_stream_free(or_stream *S)
+{
+    if (!S) return;
+    free(S->rows1); free(S->dig_M1); free(S->dig_G1); free(S->M1k);
+    free_groups(&S->G1k);
+    free(S->s1p_group); free(S->M2k);
+    free_groups(&S->G2k);
+    free(S->dig_G2k);
+    free(S);
+}
+
+/* Plain accessors (oracle/__init__.py). */
+int32_t or_st_status(const or_stream *S) { return S->status; }
+void or_st_counts(const or_stream *S, int64_t out[5])
+{
+    out[0] = S->n_e; out[1] = S->groups1; out[2] = S->pairs1; out[3] = S->n_s1p; out[4] = S->e2;
+}
+const uint32_t *or_st_rows1(const or_stream *S) { return S->rows1; }
+const uint64_t *or_st_dig(const or_stream *S, int32_t which)
+{
+    return which == 0 ? S->dig_M1 : which == 1 ? S->dig_G1 : S->dig_G2k;
+}
+const uint64_t *or_st_M(const or_stream *S, int32_t level) { return level == 1 ? S->M1k : S->M2k; }
+const int64_t *or_st_s1p_group(const or_stream *S) { return S->s1p_group; }
+static const or_groups *st_pick(const or_stream *S, int32_t level) { return level == 1 ? &S->G1k : &S->G2k; }
+int64_t or_st_g_ngroups(const or_stream *S, int32_t level) { return st_pick(S, level)->ngroups; }
+int64_t or_st_g_npairs(const or_stream *S, int32_t level) { return st_pick(S, level)->npairs; }
+const int64_t *or_st_g_trial_goffs(const or_stream *S, int32_t level) { return st_pick(S, level)->trial_goffs; }
+const uint64_t *or_st_g_ids(const or_stream *S, int32_t level) { return st_pick(S, level)->ids; }
+const int64_t *or_st_g_offs(const or_stream *S, int32_t level) { return st_pick(S, level)->offs; }
+const uint32_t *or_st_g_members(const or_stream *S, int32_t level) { return st_pick(S, level)->members; }

@@ -510,3 +510,53 @@ def test_components_vs_bfs():
     # an asymmetric CSR (edge 0 -> 3 stored once) still joins 0 and 3
     lab, k = oracle.connected_components(np.array([0, 1, 1, 1, 1]), np.array([3], np.int32))
     assert lab.tolist() == [0, 1, 2, 0] and k == 3
+
+
+@pytest.mark.parametrize("s1,c1,s2,c2,keep1,keep2", [
+    (2, 20, 2, 17, [0, 5, 19], [0, 3, 16]),
+    (3, 9, 2, 7, [8], [0, 6]),
+    (1, 6, 3, 5, [], [2]),
+])
+def test_trial_outer_stream_equals_full_run(s1, c1, s2, c2, keep1, keep2):
+    """The trial-outer streaming run (the large-config parity oracle) equals the
+    full run's corresponding trials element by element, and its per-trial
+    digests equal the digests of the full run's arrays (grouping is per trial,
+    P:L404-407, AMB-5; loop order does not change outputs)."""
+    import digests as D
+    g = SG.make("tiny")
+    args = (s1, c1, 101, s2, c2, 102)
+    ref = oracle.shingling(g.row_ptr, g.col, *args)
+    st = oracle.shingling_stream(g.row_ptr, g.col, *args, keep1=keep1, keep2=keep2)
+    assert st.counts == dict(n_e=len(ref.rows1), groups1=len(ref.G1.ids), pairs1=len(ref.G1.members),
+                             s1p=len(ref.s1p_group),
+                             entries2=int(np.diff(ref.G1.offs)[ref.s1p_group].sum()))
+    assert np.array_equal(st.rows1, ref.rows1)
+    assert np.array_equal(st.s1p_group, ref.s1p_group)
+    assert np.array_equal(st.M1k, ref.M1[:, st.keep1])
+    assert np.array_equal(st.M2k, ref.M2[:, st.keep2])
+    assert [int(x) for x in st.dig_M1] == [D.column(ref.M1[:, j]) for j in range(c1)]
+    assert [int(x) for x in st.dig_G1] == D.grouped_trials(ref.G1.trial_goffs, ref.G1.ids, ref.G1.offs,
+                                                           ref.G1.members)
+    d2 = D.grouped_trials(ref.G2.trial_goffs, ref.G2.ids, ref.G2.offs, ref.G2.members)
+    assert [int(x) for x in st.dig_G2k] == [d2[t] for t in st.keep2]
+    for G, Gk, keep in ((ref.G1, st.G1k, st.keep1), (ref.G2, st.G2k, st.keep2)):
+        for i, j in enumerate(keep):
+            a, b = G.trial_goffs[j], G.trial_goffs[j + 1]
+            a2, b2 = Gk.trial_goffs[i], Gk.trial_goffs[i + 1]
+            assert np.array_equal(G.ids[a:b], Gk.ids[a2:b2])
+            assert np.array_equal(np.diff(G.offs[a:b + 1]), np.diff(Gk.offs[a2:b2 + 1]))
+            assert np.array_equal(G.members[G.offs[a]:G.offs[b]], Gk.members[Gk.offs[a2]:Gk.offs[b2]])
+
+
+def test_digest_detects_a_moved_member():
+    """The digests are position-sensitive: swapping two members, moving a group
+    boundary, or changing one id changes the digest."""
+    import digests as D
+    ids = np.array([5, 9, 2], np.uint64)
+    offs = np.array([0, 2, 3, 5], np.int64)
+    mem = np.array([1, 4, 3, 0, 7], np.uint32)
+    d = D.grouped_trial(ids, offs, mem)
+    assert d != D.grouped_trial(ids, offs, mem[[1, 0, 2, 3, 4]])
+    assert d != D.grouped_trial(ids, np.array([0, 1, 3, 5], np.int64), mem)
+    assert d != D.grouped_trial(np.array([5, 9, 3], np.uint64), offs, mem)
+    assert D.column(np.array([1, 2], np.uint64)) != D.column(np.array([2, 1], np.uint64))
