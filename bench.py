@@ -142,46 +142,73 @@ def cpu_model():
 
 
 # ---------------------------------------------------------------- roofline
-# ncu-measured DRAM traffic per pair of the level-II kernels on gos2m (c2 = 64
-# capture, profiles/round1_gos2m_v5_ncu_full.md): hist 21.36 GB, scatter
-# 69.80 GB, fine split 92.96 GB, warp-tier local sort 43.23 GB for 2.588e9 pairs
-NCU_BYTES_PER_PAIR = {"hist2": 8.25, "scatter2": 26.97, "fine2": 35.92, "local2": 16.70}
+def int_peak(pk):
+    """Integer-ALU peak for the min-hash stages: the measured rate of the
+    hash's SASS mix (tools/int_peak.cu, profiles/int_peak.json) if present,
+    else the issue limit 128 thread-instr/clk/SM x 148 SMs x max SM clock."""
+    p = os.path.join(ROOT, "profiles", "int_peak.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hash_mix_tinstr_per_s"]), "measured (profiles/int_peak.json: " + d.get("how", "") + ")"
+    return 148 * 128 * pk["sm_max_mhz"] * 1e6 / 1e12, "derived issue limit (148 SMs x 128 instr/clk x max clock)"
+
 
 def roofline_table(stage_ms: dict, counts: dict, work: dict, pk: dict):
-    """Per-kernel algorithmic work / device time."""
+    """Algorithmic work per stage / device time.
+
+    Grouping (a5, a8): 24 B/pair (read and write a 12-B pair once) + 8 B/pair
+    run-length read of the keys + 8 B/group offsets = 32 P + 8 G bytes, over
+    the whole grouping stage (all its kernels).  Min-hash (a3, a7): 7 thread
+    instructions per (entry, trial) (the hash's SASS minimum + the compare).
+    Per-kernel rows use the kernels' own bytes (hist 8, scatter 20, local
+    16.125 B/pair)."""
     hbm = pk["hbm"]
-    issue_peak = 148 * 128 * pk["sm_max_mhz"] * 1e6 / 1e12     # T thread-instr/s
-    P1, P2 = counts["pairs1"], counts["pairs2"]
+    ipk, isrc = int_peak(pk)
+    P = {1: counts["pairs1"], 2: counts["pairs2"]}
+    G = {1: counts["groups1"], 2: counts["groups2"]}
     rows = {}
 
-    def hbm_row(stage, nbytes):
+    def hbm_row(stage, nbytes, basis):
         t = stage_ms.get(stage, 0.0) / 1e3
         if t <= 0:
             return None
         a = nbytes / t / 1e9
         return {"bound": "hbm", "achieved": round(a, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(a / hbm, 4), "ms": round(stage_ms[stage], 3), "bytes": int(nbytes)}
+                "frac": round(a / hbm, 4), "ms": round(stage_ms[stage], 3), "bytes": int(nbytes),
+                "basis": basis}
 
     def alu_row(stage, entry_trials):
         t = stage_ms.get(stage, 0.0) / 1e3
         if t <= 0:
             return None
-        a = 7.0 * entry_trials / t / 1e12                      # 7 algorithmic instr / (entry, trial)
-        return {"bound": "alu", "achieved": round(a, 3), "peak": round(issue_peak, 2),
-                "unit": "T instr/s", "frac": round(a / issue_peak, 4), "ms": round(stage_ms[stage], 3),
-                "entry_trials": int(entry_trials)}
+        a = 7.0 * entry_trials / t / 1e12
+        return {"bound": "alu", "achieved": round(a, 3), "peak": round(ipk, 2), "unit": "T instr/s",
+                "frac": round(a / ipk, 4), "ms": round(stage_ms[stage], 3),
+                "entry_trials": int(entry_trials), "basis": "7 instr per (entry, trial)", "peak_source": isrc}
 
     rows["hash1"] = alu_row("hash1", work["et1"])
     rows["hash2"] = alu_row("hash2", work["et2"])
-    for lv, P in ((1, P1), (2, P2)):
-        # hist+offsets: read 8 B key/pair; scatter: read 8 B key + write 12 B pair;
-        # local: read 12 B pair + write 4 B member + 1 head bit per pair
-        rows[f"hist{lv}"] = hbm_row(f"hist{lv}", 8 * P)
-        rows[f"scatter{lv}"] = hbm_row(f"scatter{lv}", 20 * P)
-        # fine split (two-level plans): read 12 B pair + write 12 B pair
-        rows[f"fine{lv}"] = hbm_row(f"fine{lv}", 24 * P)
-        rows[f"local{lv}"] = hbm_row(f"local{lv}", 16.125 * P)
+    for lv in (1, 2):
+        rows[f"group{lv}"] = hbm_row(f"group{lv}", 32 * P[lv] + 8 * G[lv],
+                                     "SURVEY 8(d): 24 B/pair + 8 B/pair RLE read + 8 B/group")
+        rows[f"hist{lv}"] = hbm_row(f"hist{lv}", 8 * P[lv], "kernel: 8 B/pair key read")
+        rows[f"scatter{lv}"] = hbm_row(f"scatter{lv}", 20 * P[lv], "kernel: 8 B read + 12 B write per pair")
+        rows[f"fine{lv}"] = hbm_row(f"fine{lv}", 24 * P[lv], "kernel (v1 only): 12 B read + 12 B write")
+        rows[f"local{lv}"] = hbm_row(f"local{lv}", 16.125 * P[lv], "kernel: 12 B read + 4 B + 1 bit write")
     return {k: v for k, v in rows.items() if v}
+
+
+def ncu_traffic(config: str, stage: str, pairs: int):
+    """DRAM bytes (read + write) of a stage from the committed ncu capture of
+    this build (profiles/ncu_traffic.json: bytes per pair per stage)."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None, None
+    d = json.load(open(p))
+    e = d.get(config, {}).get(stage)
+    if not e:
+        return None, None
+    return int(e["bytes_per_pair"] * pairs), e.get("source")
 
 
 # ---------------------------------------------------------------- our arm
@@ -197,12 +224,13 @@ def bench_ours(args, rank, world, local_rank):
     s1, c1, seed1, s2, c2, seed2 = (cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
     stream = torch.cuda.Stream()           # a non-default stream shared with the library
     torch.cuda.set_stream(stream)
-    dinfo = {"rank": rank, "world": world, "device": local_rank, "stream": stream.cuda_stream}
-    if dist_on:
-        uid = [None]
-        if rank == 0:
-            uid[0] = B.nccl_unique_id()
-        torch.distributed.broadcast_object_list(uid, src=0)
+    dinfo = {"rank": rank, "world": world, "device": local_rank, "stream": stream.cuda_stream,
+             "exchange": args.exchange}
+    if dist_on or args.exchange:
+        # one communicator for the whole run (one ncclUniqueId per communicator)
+        uid = [B.nccl_unique_id() if rank == 0 else None]
+        if dist_on:
+            torch.distributed.broadcast_object_list(uid, src=0)
         dinfo["nccl_uid"] = uid[0]
     # pinned host copy of the input (used by the e2e leg)
     rp_pin = torch.from_numpy(g.row_ptr).pin_memory()
@@ -219,6 +247,13 @@ def bench_ours(args, rank, world, local_rank):
     def barrier():
         if dist_on:
             torch.distributed.barrier()
+
+    def max_over_ranks(v):
+        if not dist_on:
+            return v
+        t = torch.tensor([v], device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return float(t.item())
 
     for _ in range(args.warmup):
         step()
@@ -237,17 +272,12 @@ def bench_ours(args, rank, world, local_rank):
         ev1.record(stream)
         torch.cuda.synchronize()
         barrier()
-    ms = ev0.elapsed_time(ev1) / args.steps
-    if dist_on:
-        t = torch.tensor([ms], device="cuda")
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
     counts = B.sg_get_counts(h)
     stage_ms = {k: v / args.steps for k, v in stage_sum.items()}
-    # algorithmic work of the two min-hash passes: entry x trial
-    deg = g.degrees()
+    # algorithmic work of the two min-hash passes: entry x trial (this rank)
+    deg = g.degrees()[counts["row_lo"]:counts["row_lo"] + counts["rows"]]
     et1 = float(deg[deg >= s1].sum()) * c1
-    et2 = float(counts["entries2"]) * c2      # pass-II entries = sum |L| over S1'
     launches = counts["launches"]              # kernels of the last step (counter reset each step)
     # Phase III on the device, outside the metric: clusters of
     # >= 20 vertices (the size the paper evaluated)
@@ -256,90 +286,94 @@ def bench_ours(args, rank, world, local_rank):
         lab20, ncl = B.report_dense_subgraphs(h, 0, 20, g.n)
         phase3 = {"ms": round(B.sg_get_stage_ms(h).get("report", 0.0), 3), "clusters_ge20": int(ncl),
                   "mode": "constituents (AMB-9)", "timed_in_metric": False}
-        # approach 1 (overlapping clusters), host-timed: both calls of
-        # the two-call pattern (sizes, then fill from the kept result)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         ooffs, _ = B.report_overlapping_clusters(h, 0, 20)
-        # Eq. 6 density of the reported clusters (>= 20 vertices); the paper's
-        # 0.75 +- 0.28 (Table IV context) is on the real GOS graph
         dmean, dsd, _ = B.sg_cluster_density(h, lab20, 20)
         phase3["density_ge20"] = {"mean": round(dmean, 4), "std": round(dsd, 4)}
         phase3["overlapping"] = {"ms_host": round((time.perf_counter() - t0) * 1e3, 3),
                                  "clusters_ge20": int(len(ooffs) - 1)}
-    B.shingle_graph_destroy(h)
 
-    # ---- e2e: the public API with host buffers, H2D + D2H inside the region
+    # ---- e2e: the public API with host buffers, H2D + D2H inside the region.
+    # Per step: shingle_graph_load (H2D of the pinned CSR + device validation)
+    # + 2 passes + 2 groupings + report_dense_subgraphs (Phase III) with the
+    # labels read back (world 1; with world > 1 the report is single-rank, so
+    # the counts are read back instead).
     e2e = None
     if not args.no_e2e:
         torch.cuda.synchronize()
         barrier()
-        t0 = time.perf_counter()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
         e0.record(stream)
+        d2h = 0
         for _ in range(args.steps):
-            hh = B.shingle_graph_create(rp_pin.numpy(), col_pin.numpy(), dist=dinfo)
-            B.shingle_pass(hh, s1, c1, seed1)
-            B.group_by_shingle(hh)
-            B.shingle_pass(hh, s2, c2, seed2)
-            B.group_by_shingle(hh)
-            res = B.sg_get_counts(hh)      # D2H of the step's result summary
-            B.shingle_graph_destroy(hh)
+            B.shingle_graph_load(h, rp_pin.numpy(), col_pin.numpy())
+            B.shingle_pass(h, s1, c1, seed1)
+            B.group_by_shingle(h)
+            B.shingle_pass(h, s2, c2, seed2)
+            B.group_by_shingle(h)
+            if world == 1:
+                labels, _ = B.report_dense_subgraphs(h, 0, 20, g.n)
+                d2h = labels.nbytes + 8
+            else:
+                B.sg_get_counts(h)
+                d2h = 128
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
         wall = (time.perf_counter() - t0) / args.steps * 1e3
-        ems = max(e0.elapsed_time(e1) / args.steps, wall)
-        if dist_on:
-            t = torch.tensor([ems], device="cuda")
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            ems = float(t.item())
+        ems = max_over_ranks(max(e0.elapsed_time(e1) / args.steps, wall))
         e2e = {"value": round(g.m / (ems / 1e3), 1), "unit": UNIT,
                "h2d_bytes_per_step": int(g.row_ptr.nbytes + g.col.nbytes) // max(world, 1),
-               "d2h_bytes_per_step": 80, "ms_per_step": round(ems, 3),
-               "includes": "create (H2D from pinned host + device CSR validation) + 2 passes + 2 groupings + counts D2H + destroy"}
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ems, 3),
+               "includes": ("shingle_graph_load (H2D from pinned host + device CSR validation) + 2 passes + "
+                            "2 groupings + " + ("report_dense_subgraphs + labels D2H" if world == 1
+                                                else "counts D2H"))}
+    B.shingle_graph_destroy(h)
 
     if rank != 0:
         if dist_on:
             torch.distributed.destroy_process_group()
         return
-    # rank 0's share of the work (vertex-range shards: ~1/world of every stage)
-    work = {"et1": et1 / world, "et2": et2 / world}
+    # this rank's share of the pass-II work: entries2 is global; vertex-range
+    # shards carry ~1/world of every stage
+    work = {"et1": et1, "et2": float(counts["entries2"]) * c2 / world}
     pk = peaks()
     rt = roofline_table(stage_ms, counts, work, pk)
-    dom_name = max(rt, key=lambda k: rt[k]["ms"]) if rt else None
+    cand = [k for k in ("hash1", "hash2", "group1", "group2") if k in rt]
+    dom_name = max(cand, key=lambda k: rt[k]["ms"]) if cand else None
     dom = dict(rt[dom_name]) if dom_name else None
     if dom:
-        dom["kernel"] = dom_name
-        # DRAM bytes (read + write) per pair of the dominant kernel, measured by
-        # `ncu --set full` on the same workload at c2 = 64 (one launch of each
-        # level-II kernel; profiles/round1_gos2m_v5_ncu_full.md), scaled to the
-        # pairs this stage processes per step
-        tr = NCU_BYTES_PER_PAIR.get(dom_name)
+        dom["kernel"] = dom_name + (" (stage: all its kernels)" if dom_name.startswith("group") else "")
         lv = dom_name[-1]
-        npairs = counts.get(f"pairs{lv}", 0)
-        dom["traffic"] = int(tr * npairs) if (tr and args.config == "gos2m") else None
-        dom["traffic_source"] = ("ncu dram__bytes_read.sum + dram__bytes_write.sum per pair "
-                                 "(profiles/round1_gos2m_v5_ncu_full.md) x pairs of the stage")
+        tr, src = ncu_traffic(args.config, dom_name, counts.get(f"pairs{lv}", 0) // max(world, 1))
+        dom["traffic"] = tr
+        dom["traffic_source"] = src
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         v, dt, u, nnz_s = run_oracle(g, cfg, args.cpu_sample_nnz)
         cpu = {"value": round(v, 1), "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"row prefix of the same graph: rows [0,{u}) with full adjacency ({nnz_s} entries, "
-                         f"{nnz_s // 2} edges), full two-pass method, {dt:.1f} s single-threaded",
+               "sample": f"row prefix of {args.config}: rows [0,{u}) with full adjacency ({nnz_s} entries, "
+                         f"{nnz_s // 2} edges), full two-pass method, {dt:.1f} s single-threaded "
+                         f"(the same sample as --impl reference)",
                "host_cpu": cpu_model(), "host_cores": os.cpu_count()}
+        cpu["tiny_full"] = oracle_tiny()
     clocks = clk.summary()
     out = {
         "metric": METRIC, "value": round(g.m / (ms / 1e3), 1), "unit": UNIT,
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": "u32/u64 (integer)", "data": "synthetic (seeded homology-like generator, synth/graphs.py)",
+        "vs_baseline": None, "dtype": "u32/u64 (integer)",
+        "data": "synthetic (seeded homology-like generator, synth/graphs.py)",
         "config": {"workload": f"{args.config}: n={g.n} m={g.m} (nnz={g.nnz}), s1={s1} c1={c1} s2={s2} c2={c2}",
                    "n_e": counts["n_e"], "groups1": counts["groups1"], "s1p": counts["s1p"],
                    "groups2": counts["groups2"], "pairs1": counts["pairs1"], "pairs2": counts["pairs2"],
-                   "l2": "inputs larger than L2 (CSR %.0f MB; per-step intermediates several GB)" % ((g.row_ptr.nbytes + g.col.nbytes) / 1e6),
-                   "parallelism": f"vertex-range shards x{world}"},
+                   "l2": "inputs larger than L2 (CSR %.0f MB; per-step intermediates tens of GB)"
+                         % ((g.row_ptr.nbytes + g.col.nbytes) / 1e6),
+                   "parallelism": f"vertex-range shards x{world}",
+                   "exchange": bool(counts["exchange"]), "comm_world": counts["world"]},
         "stage_ms": {k: round(v, 3) for k, v in stage_ms.items() if v > 0},
         "roofline": dom, "roofline_stages": rt, "peak_source": pk["src"], "phase3": phase3,
         "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches * args.steps,
@@ -349,6 +383,18 @@ def bench_ours(args, rank, world, local_rank):
     print(json.dumps(out))
     if dist_on:
         torch.distributed.destroy_process_group()
+
+
+def oracle_tiny():
+    """The oracle on the whole tiny config (BASELINE configs[0]), 1 core."""
+    import oracle
+    g = SG.make("tiny", cache=False)
+    c = SG.CONFIGS["tiny"]
+    t0 = time.perf_counter()
+    oracle.shingling(g.row_ptr, g.col, c["s1"], c["c1"], c["seed1"], c["s2"], c["c2"], c["seed2"])
+    dt = time.perf_counter() - t0
+    return {"value": round(g.m / dt, 1), "unit": UNIT, "seconds": round(dt, 2),
+            "workload": f"tiny: n={g.n} m={g.m}, s1=s2=2, c1=c2=100 (whole config)"}
 
 
 # ---------------------------------------------------------------- reference arm
@@ -370,10 +416,49 @@ def bench_reference(args, rank, world):
            "config": {"workload": f"{args.config} (row-prefix sample: {nnz_s} of {g.nnz} entries)"},
            "impl": "reference",
            "cpu_baseline": {"value": round(v, 1), "unit": UNIT, "cores": 1, "kind": "oracle",
-                            "sample": f"rows [0,{u}) of {args.config} with full adjacency ({nnz_s} entries)",
-                            "host_cpu": cpu_model(), "host_cores": os.cpu_count()},
+                            "sample": f"row prefix of {args.config}: rows [0,{u}) with full adjacency "
+                                      f"({nnz_s} entries), full two-pass method, median of {args.steps} "
+                                      f"steps (the same sample as our arm's cpu_baseline)",
+                            "host_cpu": cpu_model(), "host_cores": os.cpu_count(),
+                            "tiny_full": oracle_tiny()},
            "e2e": {"value": round(v, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out))
+
+
+def spawn(args_list, n):
+    """--gpus N without a torchrun environment: re-launch this script as N
+    ranks (one process per GPU) with torch.distributed.run on 127.0.0.1."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + args_list
+    return subprocess.call(cmd)
+
+
+def bench_dry(args, rank, world):
+    """--dry-run: the launch / rendezvous / max-over-ranks / JSON-line logic on
+    CPU (gloo), without the CUDA library (a CPU box can check it)."""
+    import torch
+    import torch.distributed as dist
+    if world > 1:
+        dist.init_process_group("gloo")
+    t0 = time.perf_counter()
+    x = 0
+    for _ in range(args.warmup + args.steps):
+        x += sum(range(10000))
+    ms = (time.perf_counter() - t0) * 1e3 / max(args.steps, 1)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "value": None, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                          "warmup": args.warmup, "ms_per_step": round(ms, 3), "dry_run": True,
+                          "comm_world": world}))
+    if world > 1:
+        dist.destroy_process_group()
 
 
 def main():
@@ -387,12 +472,19 @@ def main():
     ap.add_argument("--no-phase3", action="store_true", help="skip the untimed Phase III reports")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-nnz", type=int, default=1_500_000)
-    ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
+    ap.add_argument("--ref-sample-nnz", type=int, default=1_500_000)
+    ap.add_argument("--exchange", action="store_true",
+                    help="N=1: route the pairs through the NCCL exchange path anyway (a 1-rank communicator)")
+    ap.add_argument("--dry-run", action="store_true", help="CPU check of the multi-rank launch logic")
     args = ap.parse_args()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(spawn(sys.argv[1:], args.gpus))
     rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    if args.impl == "reference":
+    if args.dry_run:
+        bench_dry(args, rank, world)
+    elif args.impl == "reference":
         bench_reference(args, rank, world)
     else:
         bench_ours(args, rank, world, local_rank)

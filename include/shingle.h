@@ -61,7 +61,12 @@ typedef struct sg_dist {
     void *stream;              /* cudaStream_t to enqueue on, or NULL */
     const uint8_t *nccl_uid;   /* 128-byte ncclUniqueId (world > 1, NCCL backend) */
     void *loopback;            /* sg_loopback* (world > 1, in-process test backend) or NULL */
+    uint32_t flags;            /* SG_DIST_EXCHANGE: run the owner-routed exchange path even */
+                               /* at world == 1 (a one-rank NCCL communicator or loopback   */
+                               /* group; exercises the multi-GPU transport on one GPU)      */
 } sg_dist;
+
+#define SG_DIST_EXCHANGE 0x1u
 
 /* ------------------------------------------------------------------------ */
 /* shingle_graph_create — ingest an unweighted G(V, E) given as adjacency   */
@@ -82,6 +87,17 @@ typedef struct sg_dist {
 SG_API sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr,
                                const int32_t *col, uint32_t flags, const sg_dist *dist,
                                sg_graph **out);
+
+/* ------------------------------------------------------------------------ */
+/* shingle_graph_load — replace the resident graph of an existing handle by  */
+/* a new CSR (same arguments and validation as create), keeping the handle's */
+/* device, stream, private memory pool and communicator: the ingest step of  */
+/* a long-lived handle that shingles one graph after another (serving).     */
+/* Frees both passes' outputs; state -> created.  world > 1: collective.    */
+/* Errors: as create.  After a failed load no graph is resident and pass     */
+/* returns SG_ESTATE until a load succeeds.                                  */
+SG_API sg_status shingle_graph_load(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr,
+                                    const int32_t *col, uint32_t flags);
 
 /* ------------------------------------------------------------------------ */
 /* shingle_pass — one shingling pass (Alg. 1).      */
@@ -223,7 +239,9 @@ SG_API const char *sg_last_error(const sg_graph *g);
 /* groups), P1 pairs, P2 pairs, state, E2 (pass-II entries = sum of |L| over */
 /* S1'), device-kernel launches since create / the last reset, trial chunks  */
 /* of pass I and of pass II (negative: keys computed inside the grouping,    */
-/* DESIGN.md §6.3), 0, 0.  Global counts are summed over ranks.  The        */
+/* DESIGN.md §6.3), world (ranks of the exchange), 1 if the owner-routed   */
+/* exchange path is on (world > 1 or SG_DIST_EXCHANGE) else 0.  Global      */
+/* counts are summed over ranks.  The                                        */
 /* environment variable SG_MEM_BUDGET (bytes, read at create) caps the HBM   */
 /* the planner assumes, to exercise the chunked paths on small graphs.      */
 /* world > 1: collective (every rank calls it; it sums the counts once per   */
@@ -243,6 +261,22 @@ SG_API sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint
 SG_API sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64_t *ids,
                         int64_t *offs, uint32_t *members, const int64_t caps[2],
                         int64_t counts[3]);
+
+/* The same for the trials [t0, t1) only (grouping is per trial, */
+/* AMB-5, so a trial range is a self-contained slice of the level; t1 = -1   */
+/* means c).  trial_goffs[t1-t0+1] and offs[G+1] are relative to the first  */
+/* group / pair of trial t0; counts <- {G, Pairs, t1 - t0}.  Lets a caller    */
+/* read G_II of a 2M- or 640M-edge graph trial by trial (tens of GB in all). */
+/* SG_EINVAL unless 0 <= t0 <= t1 <= c.                                      */
+SG_API sg_status sg_get_groups_range(sg_graph *g, int32_t level, int32_t t0, int32_t t1,
+                                     int64_t *trial_goffs, uint64_t *ids, int64_t *offs,
+                                     uint32_t *members, const int64_t caps[2], int64_t counts[3]);
+
+/* Shingle matrix columns [t0, t1) of pass `level`: ids[rows x (t1-t0)]      */
+/* row-major (t1 = -1 means c); rowid as in sg_get_shingles.                 */
+SG_API sg_status sg_get_shingles_range(sg_graph *g, int32_t level, int32_t t0, int32_t t1,
+                                       uint64_t *ids, uint32_t *rowid, int64_t cap_rows,
+                                       int64_t *rows, int32_t *c);
 
 /* The S1' map: s1p_group[k] = index (in this rank's G_I, canonical order)   */
 /* of first-level shingle k; first global index of this rank in *k0.        */

@@ -36,7 +36,11 @@ class SGError(RuntimeError):
 
 class sg_dist(C.Structure):
     _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("device", C.c_int32),
-                ("stream", C.c_void_p), ("nccl_uid", C.c_void_p), ("loopback", C.c_void_p)]
+                ("stream", C.c_void_p), ("nccl_uid", C.c_void_p), ("loopback", C.c_void_p),
+                ("flags", C.c_uint32)]
+
+
+SG_DIST_EXCHANGE = 0x1
 
 
 _lib = None
@@ -54,6 +58,7 @@ def lib() -> C.CDLL:
     st = C.c_int
     sig = {
         "shingle_graph_create": (st, [i64, i64, vp, vp, u32, vp, C.POINTER(vp)]),
+        "shingle_graph_load": (st, [vp, i64, i64, vp, vp, u32]),
         "shingle_pass": (st, [vp, i32, i32, u64]),
         "group_by_shingle": (st, [vp]),
         "report_dense_subgraphs": (st, [vp, i32, i32, vp, vp]),
@@ -67,6 +72,8 @@ def lib() -> C.CDLL:
         "sg_get_counts": (st, [vp, vp]),
         "sg_get_shingles": (st, [vp, i32, vp, vp, i64, vp, vp]),
         "sg_get_groups": (st, [vp, i32, vp, vp, vp, vp, vp, vp]),
+        "sg_get_groups_range": (st, [vp, i32, i32, i32, vp, vp, vp, vp, vp, vp]),
+        "sg_get_shingles_range": (st, [vp, i32, i32, i32, vp, vp, i64, vp, vp]),
         "sg_get_s1p": (st, [vp, vp, i64, vp, vp]),
         "sg_get_hash_params": (st, [vp, i32, vp, vp, i32]),
         "sg_get_stage_ms": (st, [vp, vp, i32, vp]),
@@ -115,7 +122,8 @@ def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dic
     dptr = None
     if dist is not None:
         d = sg_dist(int(dist.get("rank", 0)), int(dist.get("world", 1)), int(dist.get("device", 0)),
-                    dist.get("stream"), None, dist.get("loopback"))
+                    dist.get("stream"), None, dist.get("loopback"),
+                    SG_DIST_EXCHANGE if dist.get("exchange") else 0)
         uid = dist.get("nccl_uid")
         if uid is not None:
             d._uid_buf = C.create_string_buffer(bytes(uid), 128)
@@ -125,6 +133,26 @@ def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dic
     rc = lib().shingle_graph_create(n, nnz, _addr(row_ptr), _addr(col), flags, dptr, C.byref(out))
     _check(rc)
     return out
+
+
+def shingle_graph_load(h, row_ptr, col, validate: bool = True):
+    """Replace the resident graph of handle h (host arrays or CUDA tensors)."""
+    dev = _is_cuda(row_ptr)
+    if not dev:
+        row_ptr = np.ascontiguousarray(row_ptr, np.int64)
+        col = np.ascontiguousarray(col, np.int32)
+    n = int(row_ptr.shape[0]) - 1
+    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE)
+    _check(lib().shingle_graph_load(h, n, int(col.shape[0]), _addr(row_ptr), _addr(col), flags), h)
+
+
+def _labels_arg(h, labels, what="labels"):
+    """int32 label array of exactly n entries (the C side reads n values)."""
+    a = np.ascontiguousarray(labels, np.int32)
+    n = sg_get_counts(h)["n"]
+    if a.ndim != 1 or len(a) != n:
+        raise ValueError(f"{what} must have n = {n} entries (got shape {a.shape})")
+    return a
 
 
 def shingle_pass(h, s: int, c: int, seed: int):
@@ -158,7 +186,7 @@ def report_overlapping_clusters(h, mode: int = 0, min_size: int = 1):
 
 def sg_cluster_density(h, labels, min_size: int = 2):
     """Eq. 6 density over the clusters of `labels`: (mean, stddev, n_clusters)."""
-    labels = np.ascontiguousarray(labels, np.int32)
+    labels = _labels_arg(h, labels)
     mean, sd, nc = C.c_double(), C.c_double(), C.c_int64()
     _check(lib().sg_cluster_density(h, labels.ctypes.data, min_size, C.byref(mean), C.byref(sd),
                                     C.byref(nc)), h)
@@ -167,8 +195,8 @@ def sg_cluster_density(h, labels, min_size: int = 2):
 
 def sg_partition_agreement(h, test_labels, bench_labels) -> dict:
     """Pair counts TP, FP, FN, TN and Eq. 2-5 (PPV, NPV, SP, SE)."""
-    t = np.ascontiguousarray(test_labels, np.int32)
-    b = np.ascontiguousarray(bench_labels, np.int32)
+    t = _labels_arg(h, test_labels, "test_labels")
+    b = _labels_arg(h, bench_labels, "bench_labels")
     cnt = np.zeros(4, np.int64)
     _check(lib().sg_partition_agreement(h, t.ctypes.data, b.ctypes.data, cnt.ctypes.data), h)
     tp, fp, fn, tn = (int(x) for x in cnt)
@@ -201,7 +229,7 @@ def sg_get_counts(h) -> dict:
     a = np.zeros(16, np.int64)
     _check(lib().sg_get_counts(h, a.ctypes.data), h)
     keys = ["n", "row_lo", "rows", "n_e", "groups1", "s1p", "groups2", "pairs1", "pairs2", "state",
-            "entries2", "launches", "chunks1", "chunks2"]
+            "entries2", "launches", "chunks1", "chunks2", "world", "exchange"]
     return dict(zip(keys, (int(x) for x in a)))
 
 
@@ -228,6 +256,34 @@ def sg_get_groups(h, level: int, with_ids: bool = True):
                                offs.ctypes.data, mem.ctypes.data, caps.ctypes.data,
                                cnt.ctypes.data), h)
     return tg, (ids if with_ids else None), offs, mem
+
+
+def sg_get_groups_range(h, level: int, t0: int, t1: int, with_ids: bool = True):
+    """Groups of trials [t0, t1) of a level; offsets relative to trial t0."""
+    cnt = np.zeros(3, np.int64)
+    _check(lib().sg_get_groups_range(h, level, t0, t1, None, None, None, None, None,
+                                     cnt.ctypes.data), h)
+    G, npairs, nt = (int(x) for x in cnt)
+    tg = np.zeros(nt + 1, np.int64)
+    ids = np.zeros(G, np.uint64)
+    offs = np.zeros(G + 1, np.int64)
+    mem = np.zeros(npairs, np.uint32)
+    caps = np.array([G, npairs], np.int64)
+    _check(lib().sg_get_groups_range(h, level, t0, t1, tg.ctypes.data,
+                                     ids.ctypes.data if with_ids else None, offs.ctypes.data,
+                                     mem.ctypes.data, caps.ctypes.data, cnt.ctypes.data), h)
+    return tg, (ids if with_ids else None), offs, mem
+
+
+def sg_get_shingles_range(h, level: int, t0: int, t1: int):
+    """Columns [t0, t1) of the shingle matrix: (ids[rows, t1-t0], rowid[rows])."""
+    rows, c = C.c_int64(), C.c_int32()
+    _check(lib().sg_get_shingles_range(h, level, t0, t1, None, None, 0, C.byref(rows), C.byref(c)), h)
+    ids = np.zeros((rows.value, t1 - t0), np.uint64)
+    rowid = np.zeros(rows.value, np.uint32)
+    _check(lib().sg_get_shingles_range(h, level, t0, t1, ids.ctypes.data, rowid.ctypes.data,
+                                       rows.value, C.byref(rows), C.byref(c)), h)
+    return ids, rowid
 
 
 def sg_get_s1p(h):

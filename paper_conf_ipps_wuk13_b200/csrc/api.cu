@@ -93,21 +93,20 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
     return;
   }
   void *p = nullptr;
-  cudaError_t e = cudaMallocAsync(&p, bytes, g->stream);
+  cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
     cache_release(g);
-    e = cudaMallocAsync(&p, bytes, g->stream);
+    e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   }
   if (e != cudaSuccess) {
     // the pool's free blocks may be too fragmented for one large request
     // (e.g. after a step with another (s, c)): return them to the device and
-    // map the request afresh
+    // map the request afresh (the handle's private pool only)
     cudaGetLastError();
     cudaStreamSynchronize(g->stream);
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, g->device) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
-    e = cudaMallocAsync(&p, bytes, g->stream);
+    cudaMemPoolTrimTo(g->pool, 0);
+    e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   }
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -261,11 +260,9 @@ struct HostMark {
 int64_t avail_bytes(sg_graph *g) {
   size_t fr = 0, tot = 0;
   CK(cudaMemGetInfo(&fr, &tot));
-  cudaMemPool_t pool;
-  CK(cudaDeviceGetDefaultMemPool(&pool, g->device));
   uint64_t reserved = 0, used = 0;
-  CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved));
-  CK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used));
+  CK(cudaMemPoolGetAttribute(g->pool, cudaMemPoolAttrReservedMemCurrent, &reserved));
+  CK(cudaMemPoolGetAttribute(g->pool, cudaMemPoolAttrUsedMemCurrent, &used));
   int64_t a = (int64_t)fr + (int64_t)(reserved - used) + g->bytes_cached - ((int64_t)1 << 30);
   if (g->mem_budget > 0) a = std::min<int64_t>(a, g->mem_budget - g->bytes_live);
   if (getenv("SG_DEBUG_MEM"))
@@ -288,7 +285,7 @@ void plan_pass_uncached(sg_graph *g, PassOut &P);
 // collective, so they are always recomputed).
 void plan_pass(sg_graph *g, PassOut &P, int level) {
   auto &m = g->plan_memo[level];
-  if (g->world == 1 && m.nrows == P.nrows && m.c == P.c && m.live == g->bytes_live &&
+  if (!g->xch && m.nrows == P.nrows && m.c == P.c && m.live == g->bytes_live &&
       m.cached == g->bytes_cached) {
     P.deferred = m.deferred;
     P.chunks.clear();
@@ -318,7 +315,7 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
   const double avail = (double)avail_bytes(g);
   int64_t ct = (int64_t)((avail - members - keys_t * c) / scr_t);
   P.deferred = false;
-  if (g->world > 1) {
+  if (g->xch) {
     // multi-rank: all keys are kept until their exchange (eager), sorted keys
     // are kept for the getters, send + receive buffers per chunk; every rank
     // uses the same trial chunks (the exchange rounds must match)
@@ -411,8 +408,11 @@ void free_scratch(sg_graph *g, GroupScratch &S) {
     dfree(g, *b);
 }
 
+bool use_group_v1();
+
 // Scratch bytes per pair of a trial segment of `maxseg` pairs (planning).
 double scratch_per_pair(int64_t maxseg) {
+  if (!use_group_v1()) return 12.5;          // v2: one partitioned copy (8 B key + 4 B value)
   int32_t b, b1;
   group_bits(maxseg, &b, &b1);
   return b == b1 ? 12.5 : 24.5;
@@ -438,8 +438,9 @@ void need(sg_graph *g, DBuf &b, size_t bytes) {
 // input order; chunks of <= group_chunk_pairs() pairs are found on the device
 // by binary search over the pieces' first chunks).  Returns the chunk count.
 int64_t build_pieces(sg_graph *g, const std::vector<Piece> &pieces, int32_t nt, GroupScratch &S,
-                     GroupPlan &plan) {
-  const int64_t CH = group_chunk_pairs();
+                     GroupPlan &plan, int64_t CH = 0) {
+  if (CH <= 0) CH = group_chunk_pairs();
+  plan.chunk = CH;
   std::vector<int32_t> tr, tc0((size_t)nt + 1, 0);
   std::vector<int64_t> in0, len, row0, c0;
   int64_t nch = 0;
@@ -568,6 +569,88 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   st_end(g, st_local);
 }
 
+// Grouping v2 (kernels_sort.cu): one stable partition by the
+// top B key bits over super-chunks, then one shared-memory sort per bucket.
+// Same contract as group_pieces.  SG_GROUP_V1=1 selects the first design
+// (A/B hook).
+bool use_group_v1() { return getenv("SG_GROUP_V1") != nullptr; }
+
+void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &pieces, int32_t t0,
+                    int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,
+                    const uint32_t *rowid, uint32_t val_base, Groups &out, uint64_t *okeys,
+                    GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter,
+                    int st_local) {
+  int64_t maxseg = 0, npairs = 0;
+  for (int j = 0; j < nt; ++j) {
+    const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
+    maxseg = std::max(maxseg, L);
+    npairs += L;
+  }
+  if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
+  int32_t bits = 0;
+  group_b_bits(maxseg, &bits);
+  const int64_t nbins = (int64_t)1 << bits;
+  GroupArgs a;
+  const int64_t nch = build_pieces(g, pieces, nt, S, a.plan, group_b_super_pairs());
+  std::vector<int64_t> seg((size_t)nt + 1);
+  for (int j = 0; j <= nt; ++j) seg[(size_t)j] = seg_all[(size_t)t0 + j];
+  upload(g, S.seg, seg.data(), seg.size() * 8);
+  need(g, S.counts, (size_t)(nch * nbins) * 4);
+  need(g, S.bstart1, (size_t)(nt * nbins) * 4);
+  need(g, S.bsize1, (size_t)(nt * nbins) * 4);
+  need(g, S.akeys, (size_t)npairs * 8);
+  need(g, S.avals, (size_t)npairs * 4);
+  need(g, S.big_list, (size_t)(nt * nbins) * 4);
+  need(g, S.big_count, 8);
+  CK(cudaMemsetAsync(S.big_count.p, 0, 8, g->stream));
+  a.plan.c = nt;
+  a.plan.bits = bits;
+  a.plan.bits1 = bits;
+  a.plan.nbins = nbins;
+  a.plan.nb1 = nbins;
+  a.plan.npairs = npairs;
+  a.plan.seg = ptr<int64_t>(S.seg);
+  if (const char *lc = getenv("SG_LOCAL_CAP")) a.plan.local_cap = atoi(lc);   // test hook
+  a.keys = keys;
+  a.vals = vals;
+  a.rowid = rowid;
+  a.val_base = val_base;
+  a.counts = ptr<uint32_t>(S.counts);
+  a.bstart1 = a.bstart = ptr<uint32_t>(S.bstart1);
+  a.bsize1 = a.bsize = ptr<uint32_t>(S.bsize1);
+  a.akeys = a.bkeys = ptr<uint64_t>(S.akeys);
+  a.avals = a.bvals = ptr<uint32_t>(S.avals);
+  a.big_list = ptr<uint32_t>(S.big_list);
+  a.big_count = ptr<uint32_t>(S.big_count);
+  a.mid_list = nullptr;
+  a.mid_count = nullptr;
+  a.members = ptr<uint32_t>(out.members);
+  a.head = ptr<uint32_t>(out.head);
+  a.okeys = okeys;
+  st_begin(g, st_hist);
+  CK(group_b_hist(a, g->stream));
+  st_end(g, st_hist);
+  st_begin(g, st_scatter);
+  CK(group_b_scatter(a, g->num_sms, g->stream));
+  if (free_after_scatter) dfree(g, *free_after_scatter);   // keys consumed
+  st_end(g, st_scatter);
+  st_begin(g, st_local);
+  CK(group_b_local(a, g->num_sms, g->stream));
+  st_end(g, st_local);
+}
+
+void group_any(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &pieces, int32_t t0,
+               int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,
+               const uint32_t *rowid, uint32_t val_base, Groups &out, uint64_t *okeys,
+               GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter, int st_local) {
+  if (use_group_v1())
+    group_pieces(g, keys, pieces, t0, nt, seg_all, vals, rowid, val_base, out, okeys, S,
+                 free_after_scatter, st_hist, st_scatter, st_local);
+  else
+    group_pieces_b(g, keys, pieces, t0, nt, seg_all, vals, rowid, val_base, out, okeys, S,
+                   free_after_scatter, st_hist, st_scatter, st_local);
+}
+
 int64_t device_sum_popc(sg_graph *g, const DBuf &words, int64_t nwords) {
   if (nwords == 0) return 0;
   DBuf d;
@@ -689,6 +772,8 @@ void owner_partition(sg_graph *g, PassOut &P, KeyChunk &ch, GroupScratch &S,
     mine->assign(bs.begin(), bs.end());
     return;
   }
+  for (int64_t v : *starts)
+    if (v > (int64_t)UINT32_MAX) fail(g, SG_EOVERFLOW, "a send buffer of one trial chunk exceeds 2^32 pairs");
   std::vector<uint32_t> st32(starts->begin(), starts->end());
   upload(g, S.bstart1, st32.data(), st32.size() * 4);
   std::vector<int64_t> zeros((size_t)nvt + 1, 0);
@@ -785,7 +870,7 @@ void group_multi(sg_graph *g, int level) {
           const int64_t len = all[k][(size_t)(s * n + (int64_t)vt * R + me)];
           if (len > 0) pieces.push_back(Piece{tl, o, len, 0});
         }
-    group_pieces(g, ptr<uint64_t>(rkeys), pieces, ch.t0, ch.nt, out.seg, ptr<uint32_t>(rvals),
+    group_any(g, ptr<uint64_t>(rkeys), pieces, ch.t0, ch.nt, out.seg, ptr<uint32_t>(rvals),
                  nullptr, 0, out, ptr<uint64_t>(out.okeys), S, nullptr,
                  level == 0 ? kStHist1 : kStHist2, level == 0 ? kStScatter1 : kStScatter2,
                  level == 0 ? kStLocal1 : kStLocal2);
@@ -796,40 +881,55 @@ void group_multi(sg_graph *g, int level) {
   g->pairs_global[level] = exchange_sum(g, out.npairs);
 }
 
-// Host view of a grouped level: per-trial group ranges, group offsets, ids.
+// Host view of trials [t0, t1) of a grouped level: per-trial group ranges,
+// group offsets (relative to the first pair of trial t0), ids.
 struct HostGroups {
   std::vector<int64_t> trial_goffs, offs;
   std::vector<uint64_t> ids;
   std::vector<uint32_t> members;
 };
 
-void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
+template <typename T>
+std::vector<T> d2h_range(sg_graph *g, const DBuf &b, size_t first, size_t count) {
+  std::vector<T> v(count);
+  if (count) {
+    CK(cudaMemcpyAsync(v.data(), reinterpret_cast<const T *>(b.p) + first, count * sizeof(T),
+                       cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+  }
+  return v;
+}
+
+void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids, int t0 = 0, int t1 = -1) {
   Groups &q = g->grp[level];
   PassOut &p = g->pass[level];
-  const int c = q.c;
-  H.members = d2h<uint32_t>(g, q.members, (size_t)q.npairs);
-  std::vector<uint32_t> head = d2h<uint32_t>(g, q.head, (size_t)((q.npairs + 31) / 32));
-  H.trial_goffs.assign((size_t)c + 1, 0);
+  if (t1 < 0) t1 = q.c;
+  const int nt = t1 - t0;
+  const int64_t p0 = q.seg[(size_t)t0], p1 = q.seg[(size_t)t1], np = p1 - p0;
+  H.members = d2h_range<uint32_t>(g, q.members, (size_t)p0, (size_t)np);
+  const int64_t w0 = p0 >> 5, w1 = (p1 + 31) >> 5;
+  std::vector<uint32_t> head = d2h_range<uint32_t>(g, q.head, (size_t)w0, (size_t)(w1 - w0));
+  H.trial_goffs.assign((size_t)nt + 1, 0);
   H.offs.clear();
   int j = 0;
-  for (int64_t i = 0; i < q.npairs; ++i) {
-    while (j < c && q.seg[(size_t)j + 1] <= i) {
+  for (int64_t i = p0; i < p1; ++i) {
+    while (j < nt && q.seg[(size_t)t0 + j + 1] <= i) {
       ++j;
       H.trial_goffs[(size_t)j] = (int64_t)H.offs.size();
     }
-    if ((head[(size_t)(i >> 5)] >> (i & 31)) & 1u) H.offs.push_back(i);
+    if ((head[(size_t)((i >> 5) - w0)] >> (i & 31)) & 1u) H.offs.push_back(i - p0);
   }
-  while (j < c) {
+  while (j < nt) {
     ++j;
     H.trial_goffs[(size_t)j] = (int64_t)H.offs.size();
   }
   const int64_t G = (int64_t)H.offs.size();
-  H.offs.push_back(q.npairs);
+  H.offs.push_back(np);
   if (!want_ids) return;
   if (q.okeys.p) {
     // multi-rank: the grouping kept the sorted keys; id = fmix^-1(key)
-    std::vector<uint64_t> ok = d2h<uint64_t>(g, q.okeys, (size_t)q.npairs);
     H.ids.resize((size_t)G);
+    std::vector<uint64_t> ok = d2h_range<uint64_t>(g, q.okeys, (size_t)p0, (size_t)np);
     for (int64_t x = 0; x < G; ++x) H.ids[(size_t)x] = fmix_inv(ok[(size_t)H.offs[(size_t)x]]);
     return;
   }
@@ -838,15 +938,64 @@ void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids) {
   if (level == 0) rid = d2h<uint32_t>(g, p.rowid, (size_t)p.nrows);
   std::vector<int64_t> rows((size_t)G);
   std::vector<int32_t> trials((size_t)G);
-  for (int jj = 0; jj < c; ++jj) {
+  for (int jj = 0; jj < nt; ++jj) {
     for (int64_t x = H.trial_goffs[(size_t)jj]; x < H.trial_goffs[(size_t)jj + 1]; ++x) {
       const uint32_t m = H.members[(size_t)H.offs[(size_t)x]];
       rows[(size_t)x] = level == 0 ? (int64_t)(std::lower_bound(rid.begin(), rid.end(), m) - rid.begin())
                                    : (int64_t)m - g->s1p_k0;
-      trials[(size_t)x] = jj;
+      trials[(size_t)x] = t0 + jj;
     }
   }
   H.ids = recompute_ids(g, level, rows, trials);
+}
+
+// Copy this rank's row range of a host (or device) CSR into HBM, rebase it
+// and validate it on the device (create and load).
+void ingest(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr, const int64_t *rp_host,
+            const int32_t *col, bool devptr, bool validate) {
+  g->n = n;
+  g->nnz_global = nnz;
+  // row range of this rank
+  std::vector<int64_t> bounds((size_t)g->world + 1);
+  if (n > 0) sg_partition_rows(n, rp_host, g->world, 8, bounds.data());
+  else std::fill(bounds.begin(), bounds.end(), 0);
+  g->row_lo = bounds[(size_t)g->rank];
+  g->row_hi = bounds[(size_t)g->rank + 1];
+  const int64_t rows = g->row_hi - g->row_lo;
+  const int64_t e0 = n > 0 ? rp_host[g->row_lo] : 0;
+  const int64_t e1 = n > 0 ? rp_host[g->row_hi] : 0;
+  // the copy below reads col[e0, e1) of the caller's buffer: check the
+  // slice on the host first (validation proper runs on the device)
+  if (e0 < 0 || e1 < e0 || e1 > nnz) fail(g, SG_EINVAL, "invalid CSR: row_ptr is not monotone within [0, nnz]");
+  g->nnz_local = e1 - e0;
+  dalloc(g, g->row_ptr, (size_t)(rows + 1) * 8);
+  dalloc(g, g->col, (size_t)g->nnz_local * 4);
+  const cudaMemcpyKind kind = devptr ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+  if (n > 0) {
+    CK(cudaMemcpyAsync(g->row_ptr.p, row_ptr + g->row_lo, (rows + 1) * 8, kind, g->stream));
+    if (g->nnz_local)
+      CK(cudaMemcpyAsync(g->col.p, col + e0, g->nnz_local * 4, kind, g->stream));
+    rebase_kernel<<<std::min<int64_t>((rows + 256) / 256, 4096), 256, 0, g->stream>>>(
+        ptr<int64_t>(g->row_ptr), rows + 1, e0);
+    CK(cudaGetLastError());
+  } else {
+    CK(cudaMemsetAsync(g->row_ptr.p, 0, 8, g->stream));
+  }
+  if (validate && rows > 0) {
+    // the CSR is validated on the device after the copy (O(nnz), one pass)
+    DBuf bad;
+    dalloc(g, bad, 4);
+    CK(cudaMemsetAsync(bad.p, 0, 4, g->stream));
+    validate_kernel<<<std::min<int64_t>((rows + 255) / 256, 8192), 256, 0, g->stream>>>(
+        ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col.p), rows,
+        g->nnz_local, n, ptr<int>(bad));
+    CK(cudaGetLastError());
+    int hb = 0;
+    CK(cudaMemcpyAsync(&hb, bad.p, 4, cudaMemcpyDeviceToHost, g->stream));
+    sync(g);
+    dfree(g, bad);
+    if (hb) fail(g, SG_EINVAL, "invalid CSR: a row is not strictly increasing, or an id is outside [0, n)");
+  }
 }
 
 }  // namespace
@@ -956,50 +1105,19 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
       g->own_stream = true;
     }
     CK(cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking));
-    // keep freed blocks cached in the pool: re-runs and resets reuse them
-    cudaMemPool_t pool;
-    CK(cudaDeviceGetDefaultMemPool(&pool, g->device));
+    // a private stream-ordered pool: freed blocks stay cached for re-runs
+    // and resets, without changing the device's default pool for other users
+    cudaMemPoolProps pp;
+    memset(&pp, 0, sizeof pp);
+    pp.allocType = cudaMemAllocationTypePinned;
+    pp.handleTypes = cudaMemHandleTypeNone;
+    pp.location.type = cudaMemLocationTypeDevice;
+    pp.location.id = g->device;
+    CK(cudaMemPoolCreate(&g->pool, &pp));
     uint64_t thr = UINT64_MAX;
-    CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
-    // row range of this rank
-    std::vector<int64_t> bounds((size_t)g->world + 1);
-    if (n > 0) sg_partition_rows(n, rp_host, g->world, 8, bounds.data());
-    else std::fill(bounds.begin(), bounds.end(), 0);
-    g->row_lo = bounds[(size_t)g->rank];
-    g->row_hi = bounds[(size_t)g->rank + 1];
-    const int64_t rows = g->row_hi - g->row_lo;
-    const int64_t e0 = n > 0 ? rp_host[g->row_lo] : 0;
-    const int64_t e1 = n > 0 ? rp_host[g->row_hi] : 0;
-    g->nnz_local = e1 - e0;
-    dalloc(g, g->row_ptr, (size_t)(rows + 1) * 8);
-    dalloc(g, g->col, (size_t)g->nnz_local * 4);
-    const cudaMemcpyKind kind = devptr ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
-    if (n > 0) {
-      CK(cudaMemcpyAsync(g->row_ptr.p, row_ptr + g->row_lo, (rows + 1) * 8, kind, g->stream));
-      if (g->nnz_local)
-        CK(cudaMemcpyAsync(g->col.p, col + e0, g->nnz_local * 4, kind, g->stream));
-      rebase_kernel<<<std::min<int64_t>((rows + 256) / 256, 4096), 256, 0, g->stream>>>(
-          ptr<int64_t>(g->row_ptr), rows + 1, e0);
-      CK(cudaGetLastError());
-    } else {
-      CK(cudaMemsetAsync(g->row_ptr.p, 0, 8, g->stream));
-    }
-    if (validate && rows > 0) {
-      // the CSR is validated on the device after the copy (O(nnz), one pass)
-      DBuf bad;
-      dalloc(g, bad, 4);
-      CK(cudaMemsetAsync(bad.p, 0, 4, g->stream));
-      validate_kernel<<<std::min<int64_t>((rows + 255) / 256, 8192), 256, 0, g->stream>>>(
-          ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col.p), rows,
-          g->nnz_local, n, ptr<int>(bad));
-      CK(cudaGetLastError());
-      int hb = 0;
-      CK(cudaMemcpyAsync(&hb, bad.p, 4, cudaMemcpyDeviceToHost, g->stream));
-      sync(g);
-      dfree(g, bad);
-      if (hb) fail(g, SG_EINVAL, "invalid CSR: a row is not strictly increasing, or an id is outside [0, n)");
-    }
-    if (g->world > 1) g->xch = exchange_create(g, dist);
+    CK(cudaMemPoolSetAttribute(g->pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, validate);
+    if (g->world > 1 || (dist && (dist->flags & SG_DIST_EXCHANGE))) g->xch = exchange_create(g, dist);
     sync(g);
     g->launch_base = g_launches.load();
     g->state = kCreated;
@@ -1018,10 +1136,43 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
     cudaGetLastError();
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
     if (g->side) cudaStreamDestroy(g->side);
+    if (g->pool) cudaMemPoolDestroy(g->pool);
+    cudaGetLastError();
     return st;
   }
   *out = G.release();
   return SG_OK;
+}
+
+sg_status shingle_graph_load(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr,
+                             const int32_t *col, uint32_t flags) {
+  return guarded(g, [&] {
+    if (n < 0 || (uint64_t)n >= kP || nnz < 0 || (n > 0 && !row_ptr) || (nnz > 0 && !col))
+      fail(g, SG_EINVAL, "invalid n / nnz / pointers (need 0 <= n < 2^31 - 1)");
+    const bool devptr = flags & SG_DEVICE_PTRS;
+    std::vector<int64_t> hrp;
+    const int64_t *rp_host = row_ptr;
+    if (devptr && n > 0) {
+      hrp.resize((size_t)n + 1);
+      CK(cudaMemcpy(hrp.data(), row_ptr, (n + 1) * 8, cudaMemcpyDeviceToHost));
+      rp_host = hrp.data();
+    }
+    if (n > 0 && (rp_host[0] != 0 || rp_host[n] != nnz))
+      fail(g, SG_EINVAL, "invalid CSR: row_ptr[0] must be 0 and row_ptr[n] must equal nnz");
+    for (int l = 0; l < 2; ++l) {
+      free_pass(g, g->pass[l]);
+      free_groups(g, g->grp[l]);
+    }
+    dfree(g, g->row_ptr);
+    dfree(g, g->col);
+    g->e2_global = -1;
+    g->ov_valid = false;
+    g->state = kEmpty;                  // until the new graph is resident and valid
+    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, !(flags & SG_NO_VALIDATE));
+    sync(g);
+    g->state = kCreated;
+    g->launch_base = g_launches.load();
+  }, true);
 }
 
 sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
@@ -1087,8 +1238,8 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
     P.key_stride = key_stride_for(nrows);
     P.blocks = {0, nrows};
     if (level == 0) {
-      g->n_e_global = g->world > 1 ? exchange_sum(g, nrows) : nrows;
-    } else if (g->world > 1) {
+      g->n_e_global = g->xch ? exchange_sum(g, nrows) : nrows;
+    } else if (g->xch) {
       assign_s1p_index(g, P);            // |S1'| global, canonical dense index per row
     } else {
       g->s1p_global = nrows;
@@ -1128,7 +1279,7 @@ sg_status group_by_shingle(sg_graph *g) {
     PassOut &P = g->pass[level];
     const int c = P.c;
     st_begin(g, level == 0 ? kStGroup1 : kStGroup2);
-    if (g->world > 1) {
+    if (g->xch) {
       group_multi(g, level);
     } else {
       Groups &out = g->grp[level];
@@ -1154,7 +1305,7 @@ sg_status group_by_shingle(sg_graph *g) {
         std::vector<Piece> pieces;
         for (int tl = 0; tl < ch.nt; ++tl)
           pieces.push_back(Piece{tl, (int64_t)tl * P.key_stride, P.nrows, 0});
-        group_pieces(g, ptr<uint64_t>(ch.keys), pieces, ch.t0, ch.nt, out.seg, nullptr, rowid, base,
+        group_any(g, ptr<uint64_t>(ch.keys), pieces, ch.t0, ch.nt, out.seg, nullptr, rowid, base,
                      out, nullptr, S, &ch.keys, level == 0 ? kStHist1 : kStHist2,
                      level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2);
         ch.computed = false;
@@ -1213,6 +1364,7 @@ void shingle_graph_destroy(sg_graph *g) {
   if (g->xch) exchange_destroy(g->xch);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   if (g->side) cudaStreamDestroy(g->side);
+  if (g->pool) cudaMemPoolDestroy(g->pool);
   cudaGetLastError();
   delete g;
 }
@@ -1227,7 +1379,7 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[16]) {
       if (grouped && g->groups_global[l] < 0) {
         Groups &q = g->grp[l];
         int64_t loc = device_sum_popc(g, q.head, (q.npairs + 31) / 32);
-        g->groups_global[l] = g->world > 1 ? exchange_sum(g, loc) : loc;
+        g->groups_global[l] = g->xch ? exchange_sum(g, loc) : loc;
       }
     }
     if (g->state >= kPassed2 && g->e2_global < 0) {
@@ -1239,7 +1391,7 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[16]) {
       CK(cudaMemcpyAsync(&h, d.p, 8, cudaMemcpyDeviceToHost, g->stream));
       sync(g);
       dfree(g, d);
-      g->e2_global = g->world > 1 ? exchange_sum(g, (int64_t)h) : (int64_t)h;
+      g->e2_global = g->xch ? exchange_sum(g, (int64_t)h) : (int64_t)h;
     }
     counts[0] = g->n;
     counts[1] = g->row_lo;
@@ -1258,31 +1410,32 @@ sg_status sg_get_counts(const sg_graph *gc, int64_t counts[16]) {
       const int64_t nch = (int64_t)P.chunks.size();
       counts[12 + l] = P.deferred ? -nch : nch;
     }
-    counts[14] = counts[15] = 0;
+    counts[14] = g->world;                    // ranks of the exchange (communicator size)
+    counts[15] = g->xch ? 1 : 0;              // owner-routed exchange path on
   }, true);
 }
 
-sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *rowid,
-                          int64_t cap_rows, int64_t *rows, int32_t *c) {
+sg_status sg_get_shingles_range(sg_graph *g, int32_t level, int32_t t0, int32_t t1, uint64_t *ids,
+                                uint32_t *rowid, int64_t cap_rows, int64_t *rows, int32_t *c) {
   return guarded(g, [&] {
     if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
     const int l = level - 1;
     if (g->state < (l == 0 ? kPassed1 : kPassed2)) fail(g, SG_ESTATE, "pass not run yet");
     PassOut &P = g->pass[l];
-    if (l == 0 && g->state >= kPassed2) {
-      // pass-I rows are still resident; entries (the CSR) too
-    }
+    if (t1 < 0) t1 = P.c;
+    if (t0 < 0 || t0 > t1 || t1 > P.c) fail(g, SG_EINVAL, "need 0 <= t0 <= t1 <= c");
     if (rows) *rows = P.nrows;
     if (c) *c = P.c;
     if (!ids && !rowid) return;
     if (cap_rows < P.nrows) fail(g, SG_EINVAL, "buffer too small");
     if (ids) {
-      std::vector<int64_t> rq((size_t)(P.nrows * P.c));
+      const int nt = t1 - t0;
+      std::vector<int64_t> rq((size_t)(P.nrows * nt));
       std::vector<int32_t> tq(rq.size());
       for (int64_t r = 0; r < P.nrows; ++r)
-        for (int j = 0; j < P.c; ++j) {
-          rq[(size_t)(r * P.c + j)] = r;
-          tq[(size_t)(r * P.c + j)] = j;
+        for (int j = 0; j < nt; ++j) {
+          rq[(size_t)(r * nt + j)] = r;
+          tq[(size_t)(r * nt + j)] = t0 + j;
         }
       std::vector<uint64_t> v = recompute_ids(g, l, rq, tq);
       if (!v.empty()) memcpy(ids, v.data(), v.size() * 8);
@@ -1306,21 +1459,31 @@ sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *r
   });
 }
 
-sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64_t *ids,
-                        int64_t *offs, uint32_t *members, const int64_t caps[2], int64_t counts[3]) {
+sg_status sg_get_shingles(sg_graph *g, int32_t level, uint64_t *ids, uint32_t *rowid,
+                          int64_t cap_rows, int64_t *rows, int32_t *c) {
+  return sg_get_shingles_range(g, level, 0, -1, ids, rowid, cap_rows, rows, c);
+}
+
+sg_status sg_get_groups_range(sg_graph *g, int32_t level, int32_t t0, int32_t t1,
+                              int64_t *trial_goffs, uint64_t *ids, int64_t *offs, uint32_t *members,
+                              const int64_t caps[2], int64_t counts[3]) {
   return guarded(g, [&] {
     if (level != 1 && level != 2) fail(g, SG_EINVAL, "level must be 1 or 2");
     const int l = level - 1;
     if (g->state < (l == 0 ? kGrouped1 : kGrouped2)) fail(g, SG_ESTATE, "not grouped yet");
+    const int c = g->grp[l].c;
+    if (t1 < 0) t1 = c;
+    if (t0 < 0 || t0 > t1 || t1 > c) fail(g, SG_EINVAL, "need 0 <= t0 <= t1 <= c");
     HostGroups H;
-    host_groups(g, l, H, ids != nullptr);
+    const bool fill = trial_goffs || ids || offs || members;
+    host_groups(g, l, H, fill && ids != nullptr, t0, t1);
     const int64_t G = (int64_t)H.offs.size() - 1;
     if (counts) {
       counts[0] = G;
       counts[1] = (int64_t)H.members.size();
-      counts[2] = g->grp[l].c;
+      counts[2] = t1 - t0;
     }
-    if (!trial_goffs && !ids && !offs && !members) return;
+    if (!fill) return;
     if (!caps || caps[0] < G || caps[1] < (int64_t)H.members.size())
       fail(g, SG_EINVAL, "buffers too small");
     if (trial_goffs) memcpy(trial_goffs, H.trial_goffs.data(), H.trial_goffs.size() * 8);
@@ -1328,6 +1491,11 @@ sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64
     if (offs) memcpy(offs, H.offs.data(), H.offs.size() * 8);
     if (members && !H.members.empty()) memcpy(members, H.members.data(), H.members.size() * 4);
   });
+}
+
+sg_status sg_get_groups(sg_graph *g, int32_t level, int64_t *trial_goffs, uint64_t *ids,
+                        int64_t *offs, uint32_t *members, const int64_t caps[2], int64_t counts[3]) {
+  return sg_get_groups_range(g, level, 0, -1, trial_goffs, ids, offs, members, caps, counts);
 }
 
 sg_status sg_get_s1p(sg_graph *g, int64_t *s1p_group, int64_t cap, int64_t *count, int64_t *k0) {
@@ -1622,7 +1790,9 @@ sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_siz
     for (int64_t r = 0; r < n; ++r) {
       const int64_t k = sz[(size_t)r];
       if (k < thr) continue;
-      const double d = (double)(e2[(size_t)r] / 2) / ((double)k * (double)(k - 1) / 2.0);
+      // each stored entry (u, v), u != v, inside the cluster is half an edge
+      // (symmetric rows: exactly the edge count; AMB-21)
+      const double d = ((double)e2[(size_t)r] / 2.0) / ((double)k * (double)(k - 1) / 2.0);
       ++c;
       s1 += d;
       s2 += d * d;

@@ -2,8 +2,11 @@
 #include <dlfcn.h>
 #include <nccl.h>
 
+#include <chrono>
 #include <condition_variable>
+#include <cstdlib>
 #include <cstring>
+#include <thread>
 #include <mutex>
 #include <vector>
 
@@ -58,6 +61,8 @@ struct NcclApi {
   decltype(&ncclGroupStart) groupStart = nullptr;
   decltype(&ncclGroupEnd) groupEnd = nullptr;
   decltype(&ncclGetErrorString) errStr = nullptr;
+  decltype(&ncclCommGetAsyncError) asyncError = nullptr;   // optional (polling)
+  decltype(&ncclCommAbort) commAbort = nullptr;            // optional (polling)
 };
 
 NcclApi *nccl_api(std::string *why) {
@@ -81,6 +86,8 @@ NcclApi *nccl_api(std::string *why) {
       api.groupStart = (decltype(api.groupStart))dlsym(api.so, "ncclGroupStart");
       api.groupEnd = (decltype(api.groupEnd))dlsym(api.so, "ncclGroupEnd");
       api.errStr = (decltype(api.errStr))dlsym(api.so, "ncclGetErrorString");
+      api.asyncError = (decltype(api.asyncError))dlsym(api.so, "ncclCommGetAsyncError");
+      api.commAbort = (decltype(api.commAbort))dlsym(api.so, "ncclCommAbort");
       ok = api.getUniqueId && api.commInitRank && api.commDestroy && api.allGather && api.send &&
            api.recv && api.groupStart && api.groupEnd && api.errStr;
     }
@@ -99,6 +106,41 @@ struct Exchange {
   void *dbuf = nullptr;      // device scratch for NCCL all-gathers
   size_t dbytes = 0;
 };
+
+// Wait for the handle's stream while polling the communicator: a peer that
+// failed (or a broken link) surfaces as an asynchronous NCCL error; the
+// communicator is then aborted so this rank returns SG_ENCCL instead of
+// hanging in a collective.  SG_NCCL_TIMEOUT_S (default 600) bounds the wait.
+static void nccl_wait(sg_graph *g, const char *what) {
+  Exchange *x = g->xch;
+  static const double limit = [] {
+    const char *e = getenv("SG_NCCL_TIMEOUT_S");
+    return e ? atof(e) : 600.0;
+  }();
+  const auto t0 = std::chrono::steady_clock::now();
+  for (int it = 0;; ++it) {
+    const cudaError_t q = cudaStreamQuery(g->stream);
+    if (q == cudaSuccess) return;
+    if (q != cudaErrorNotReady) ck(g, q, what);
+    if (x->nccl->asyncError) {
+      ncclResult_t ae = ncclSuccess;
+      if (x->nccl->asyncError(x->comm, &ae) == ncclSuccess && ae != ncclSuccess && ae != ncclInProgress) {
+        if (x->nccl->commAbort) x->nccl->commAbort(x->comm);
+        x->comm = nullptr;
+        fail(g, SG_ENCCL, std::string(what) + ": asynchronous NCCL error: " + x->nccl->errStr(ae));
+      }
+    }
+    if (it > 2000) {
+      std::this_thread::sleep_for(std::chrono::microseconds(50));
+      const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+      if (el > limit) {
+        if (x->nccl->commAbort) x->nccl->commAbort(x->comm);
+        x->comm = nullptr;
+        fail(g, SG_ENCCL, std::string(what) + ": timed out (SG_NCCL_TIMEOUT_S); communicator aborted");
+      }
+    }
+  }
+}
 
 static void nck(sg_graph *g, ncclResult_t r, const char *what) {
   if (r != ncclSuccess) {
@@ -171,9 +213,10 @@ void x_allgather_i64(sg_graph *g, const int64_t *mine, int64_t n, int64_t *all) 
   int64_t *din = reinterpret_cast<int64_t *>(x->dbuf);
   int64_t *dout = din + n;
   ck(g, cudaMemcpyAsync(din, mine, (size_t)n * 8, cudaMemcpyHostToDevice, g->stream), "H2D");
+  if (!x->comm) fail(g, SG_ENCCL, "communicator was aborted");
   nck(g, x->nccl->allGather(din, dout, (size_t)n, ncclInt64, x->comm, g->stream), "ncclAllGather");
   ck(g, cudaMemcpyAsync(all, dout, (size_t)n * 8 * x->world, cudaMemcpyDeviceToHost, g->stream), "D2H");
-  ck(g, cudaStreamSynchronize(g->stream), "sync");
+  nccl_wait(g, "ncclAllGather");
 }
 
 int64_t exchange_sum(sg_graph *g, int64_t v) {
@@ -214,6 +257,7 @@ void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
     lb_barrier(g, lb);                                        // senders may reuse buffers
     return;
   }
+  if (!x->comm) fail(g, SG_ENCCL, "communicator was aborted");
   nck(g, x->nccl->groupStart(), "ncclGroupStart");
   for (int p = 0; p < R; ++p) {
     const int64_t sc = soff[p + 1] - soff[p], rc = roff[p + 1] - roff[p];
@@ -225,7 +269,7 @@ void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
                            g->stream), "ncclRecv");
   }
   nck(g, x->nccl->groupEnd(), "ncclGroupEnd");
-  ck(g, cudaStreamSynchronize(g->stream), "sync");
+  nccl_wait(g, "ncclSend/ncclRecv");
 }
 
 }  // namespace sg

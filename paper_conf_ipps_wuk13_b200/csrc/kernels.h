@@ -72,6 +72,8 @@ struct GroupPlan {
   int64_t *chunk_in0 = nullptr;    // [nchunks] key / explicit-value index of the chunk's first pair
   int64_t *seg = nullptr;          // [c+1] output position of pair 0 of trial j (global)
   int32_t *trial_chunk0 = nullptr; // [c+1] first chunk of each trial
+  int64_t chunk = 4096;            // pairs per chunk (the tables above)
+  int32_t local_cap = 0;           // grouping v2: largest bucket sorted in shared memory (0: default)
 };
 
 struct GroupArgs {
@@ -126,6 +128,21 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level 
 // Sort every final bucket and write members + head bits: warp tier, then the
 // mid and big tiers over the lists the warp tier filled (no host sync).
 cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
+// Global-memory sort of the buckets listed in big_list (count on the device).
+cudaError_t group_big(const GroupArgs &g, int num_sms, cudaStream_t st);
+
+// ---- grouping v2 (kernels_sort.cu): one stable partition by
+// the top `plan.bits` (<= 13) key bits over super-chunks of
+// group_b_super_pairs() pairs (plan.chunk), then a shared-memory sort per
+// bucket.  Single level: plan.nbins = plan.nb1 = 2^bits, bkeys = akeys,
+// bvals = avals, bstart = bstart1, bsize = bsize1.
+int64_t group_b_super_pairs();
+int32_t group_b_max_bits();
+int32_t group_b_local_cap();
+void group_b_bits(int64_t maxseg, int32_t *bits);
+cudaError_t group_b_hist(const GroupArgs &g, cudaStream_t st);       // + offsets
+cudaError_t group_b_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
+cudaError_t group_b_local(const GroupArgs &g, int num_sms, cudaStream_t st);   // + big
 
 // ---- Phase III on the device (kernels_report.cu) ---------------------------
 struct ReportArgs {

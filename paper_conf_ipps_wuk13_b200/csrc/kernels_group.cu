@@ -399,10 +399,10 @@ __global__ void chunk_table_kernel(const int32_t *__restrict__ p_trial,
       if (p_chunk0[mid] <= k) lo = mid;
       else hi = mid;
     }
-    const int64_t a = (k - p_chunk0[lo]) * kChunk;
+    const int64_t a = (k - p_chunk0[lo]) * plan.chunk;
     plan.chunk_i0[k] = p_row0[lo] + a;
     plan.chunk_in0[k] = p_in0[lo] + a;
-    plan.chunk_len[k] = (int32_t)min((int64_t)kChunk, p_len[lo] - a);
+    plan.chunk_len[k] = (int32_t)min(plan.chunk, p_len[lo] - a);
     plan.chunk_trial[k] = p_trial[lo];
   }
 }

@@ -554,6 +554,10 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   // big tier (length read on the device)
+  return group_big(g, num_sms, st);
+}
+
+cudaError_t group_big(const GroupArgs &g, int num_sms, cudaStream_t st) {
   big_kernel<<<num_sms, 1024, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();

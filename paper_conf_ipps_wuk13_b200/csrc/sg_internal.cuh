@@ -61,6 +61,7 @@ __device__ __forceinline__ uint32_t m31_hash(uint32_t A, uint32_t B, uint32_t v)
 // Handle
 // ----------------------------------------------------------------------------
 enum State : int32_t {
+  kEmpty = -1,    // a shingle_graph_load failed: no valid graph resident
   kCreated = 0,   // CSR resident
   kPassed1 = 1,   // pass I rows selected (keys computed unless deferred)
   kGrouped1 = 2,  // G_I resident
@@ -143,7 +144,8 @@ struct sg_graph {
   bool own_stream = false;
   cudaStream_t side = nullptr;     // min-hash of later trial chunks, overlapped with grouping
   int32_t rank = 0, world = 1;
-  sg::Exchange *xch = nullptr;
+  sg::Exchange *xch = nullptr;      // owner-routed exchange path (world > 1, or SG_DIST_EXCHANGE)
+  cudaMemPool_t pool = nullptr;     // the handle's private stream-ordered pool
   int num_sms = 148;
   // graph (global n; this rank's rows [row_lo, row_hi))
   int64_t n = 0, nnz_global = 0;

@@ -257,6 +257,12 @@ CONFIGS = {
     "hub2m": dict(gen=dict(n=2_000_000, n_isolated=437_016, m_target=56_919_738, fam_hi=3000,
                            n_hubs=20_000),
                   seed=3, s1=2, c1=200, seed1=301, s2=2, c2=200, seed2=302),
+    # configs[3]: Pacific-Ocean-shaped 11M vertices / 640M edges (P:L71-74,
+    # P:L1316-1321): the config-2 recipe scaled (same singleton share,
+    # family and component size laws); s1=2, c1=200, s2=2, c2=100 (P:L843-845,
+    # AMB-20)
+    "pacific640m": dict(gen=dict(n=11_000_000, n_isolated=2_403_588, m_target=640_000_000, fam_hi=3000),
+                        seed=4, s1=2, c1=200, seed1=401, s2=2, c2=100, seed2=402),
     # small variants for parity tests (same recipe, oracle-sized)
     "small": dict(gen=dict(n=60_000, n_isolated=13_000, m_target=1_700_000, n_cliques=20,
                            cc_max=10_707, fam_hi=600),

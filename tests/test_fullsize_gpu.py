@@ -3,10 +3,12 @@ vertices, 56.9M edges, s1 = s2 = 2, c1 = c2 = 200), in the launch
 configuration bench.py times (one GPU, the same trial chunking).
 
 The oracle cannot run the whole method at this size in seconds, so the checks
-are (a) sampled outputs the oracle computes one by one (pass-I shingle rows)
-and (b) properties that hold at any size: the selected rows, the canonical
-order of G_I, each sampled group's members sharing its id, the S1' filter,
-and the pair / entry counts of both levels.
+are (a) sampled outputs the oracle computes one by one (pass-I shingle rows),
+(b) properties that hold at any size: the selected rows, the canonical order
+of G_I, each sampled group's members sharing its id, the S1' filter, and the
+pair / entry counts of both levels, and (c) digests written by the oracle's
+trial-outer run (tools/oracle_digests.py): every pass-I column and G_I trial,
+and four full pass-II columns / G_II trials.
 """
 import numpy as np
 import pytest
@@ -56,8 +58,10 @@ def run():
     lab_s = np.where(np.isin(labels, pick), labels, np.arange(g.n, dtype=np.int32)).astype(np.int32)
     out["lab_s"] = lab_s
     out["dens_s"] = B.sg_cluster_density(h, lab_s, 2)
+    out["handle2"] = h            # G_II stays resident for the per-trial digest test
+    out["B"] = B
+    yield g, cfg, out
     B.shingle_graph_destroy(h)
-    return g, cfg, out
 
 
 def test_fullsize_rows_and_sampled_pass1_shingles(run):
@@ -176,3 +180,41 @@ def test_fullsize_density(run):
     assert abs(mean - rm) <= 1e-12 and abs(sd - rs) <= 1e-12
     mean, sd, nc = out["dens20"]
     assert nc == out["nc20"] and 0.0 < mean <= 1.0 and 0.0 <= sd <= 0.5
+
+
+@pytest.mark.timeout(1800)
+def test_fullsize_digests_every_pass1_trial_and_sampled_pass2_trials(run):
+    """Bit-exact parity at full size (gos2m, the bench workload) against the
+    oracle's trial-outer run (tests/golden/digests_gos2m.json, written by
+    tools/oracle_digests.py): every pass-I column and every G_I trial by
+    digest, the S1' map, and the pass-II columns and G_II trials 0, 63, 64
+    and 199 (the first / last trial of the first chunk, the first of the
+    second chunk, the last trial) with their G_II trials read one at a time."""
+    import json
+    import os
+
+    import digests as D
+    g, cfg, out = run
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "digests_gos2m.json")))
+    assert gold["graph_digest"] == D.column(np.concatenate([g.row_ptr.astype(np.uint64),
+                                                           g.col.astype(np.uint64)])), \
+        "generator produced another graph than the one the digests were written for"
+    c = out["counts"]
+    for k in ("n_e", "groups1", "pairs1", "s1p", "entries2"):
+        assert c[k] == gold["counts"][k], k
+    ids1, rows1 = out["M1"]
+    assert D.column(rows1.astype(np.uint64)) == gold["rows1_digest"]
+    for j in range(cfg["c1"]):
+        assert D.column(np.ascontiguousarray(ids1[:, j])) == gold["dig_M1"][j], f"pass-I column {j}"
+    tg, gid, offs, mem = out["G1"]
+    assert D.grouped_trials(tg, gid, offs, mem) == gold["dig_G1"]
+    s1p, _ = out["s1p"]
+    assert D.column(s1p.astype(np.uint64)) == gold["s1p_digest"]
+    h = out["handle2"]
+    B = out["B"]
+    for i, t in enumerate(gold["keep2"]):
+        m2, _ = B.sg_get_shingles_range(h, 2, t, t + 1)
+        assert D.column(np.ascontiguousarray(m2[:, 0])) == gold["dig_M2k"][i], f"pass-II column {t}"
+        tg2, gid2, offs2, mem2 = B.sg_get_groups_range(h, 2, t, t + 1)
+        assert len(gid2) == gold["G2k_groups"][i]
+        assert D.grouped_trial(gid2, offs2, mem2) == gold["dig_G2k"][i], f"G_II trial {t}"

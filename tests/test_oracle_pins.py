@@ -468,6 +468,17 @@ def test_density_closed_forms():
     assert nc == 1 and math.isclose(mean, 2 / 6)
     mean, _, nc = oracle.cluster_density(rp, col, lab2)
     assert nc == 3 and math.isclose(mean, (0.4 + 0.4 + 2 / 6) / 3)
+    # a self-loop is not an edge between two vertices of the cluster (AMB-21):
+    # the 2-vertex cluster {0, 1} with one edge and two self-loops has density 1
+    rp3 = np.array([0, 2, 4], np.int64)
+    col3 = np.array([0, 1, 0, 1], np.int32)
+    mean, _, nc = oracle.cluster_density(rp3, col3, np.array([0, 0]))
+    assert nc == 1 and mean == 1.0
+    # a one-directional entry counts half an edge: {0, 1, 2}, entries 0->1, 1->0, 1->2
+    rp4 = np.array([0, 1, 3, 3], np.int64)
+    col4 = np.array([1, 0, 2], np.int32)
+    mean, _, _ = oracle.cluster_density(rp4, col4, np.array([0, 0, 0]))
+    assert math.isclose(mean, 1.5 / 3)
 
 
 # ---------------------------------------------------------------- Eq. 2-5 pair counts

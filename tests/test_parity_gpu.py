@@ -98,7 +98,8 @@ def test_small_homology_parity(B):
 
 
 def test_hub_rows_longer_than_staging_buffer(B):
-    """Rows of 5K-12K entries exceed the per-warp smem stage (chunked path)."""
+    """Rows of 5K-12K entries: longer than 2,048 entries, so pass I takes them
+    with the block-per-vertex hub_kernel (staged once, < 16,384 entries)."""
     g = SG.make("hubsmall")
     assert g.degrees().max() > 4096
     cfg = SG.CONFIGS["hubsmall"]
@@ -108,11 +109,81 @@ def test_hub_rows_longer_than_staging_buffer(B):
 
 def test_big_bucket_path_large_clique(B):
     """A 5,000-clique: in every trial ~4,998 vertices share one shingle, a
-    group larger than the 4,096-element shared-memory bucket (global path)."""
+    group of ~5K generators in one bucket."""
     g = SG.cliques([5000, 30, 12], n=6000, seed=3)
     out, ref = run_both(B, g, 2, 6, 11, 2, 5, 12)
     assert_parity(out, ref)
     assert np.diff(ref.G1.offs).max() > 4096
+
+
+@pytest.mark.parametrize("cap", ["64", "1024"])
+def test_oversize_buckets_take_the_global_sort(B, cap, monkeypatch):
+    """SG_LOCAL_CAP shrinks the shared-memory bucket sort's capacity so that
+    buckets holding big groups (the 5,000-clique) and ordinary ones overflow
+    into the global-memory sort (big_kernel)."""
+    monkeypatch.setenv("SG_LOCAL_CAP", cap)
+    g = SG.cliques([5000, 300, 30, 12], n=6000, seed=4)
+    out, ref = run_both(B, g, 2, 7, 13, 2, 6, 14)
+    assert_parity(out, ref)
+
+
+def branch_graph():
+    """Complete bipartite blocks K_{a,3}: the 3 right vertices of a block have
+    rows of exactly a entries (pass I) and its a left vertices share every
+    first-level shingle, i.e. one G_I group of a generators per trial, which
+    is a pass-II row of exactly a entries.  The lengths straddle every
+    min-hash branch: <= 8 (paired short rows), 24, the per-warp stage (512 /
+    1,024 entries), the 2,048 hub threshold and the 16,384-entry hub stage."""
+    sizes = [1, 2, 5, 8, 9, 24, 25, 511, 512, 513, 1023, 1024, 1025, 2047, 2048, 2049,
+             16383, 16384, 16385, 40000]
+    n = sum(sizes) + 3 * len(sizes) + 500
+    rng = np.random.default_rng(9)
+    perm = rng.permutation(n).astype(np.int64)
+    a_list, b_list, base = [], [], 0
+    for a in sizes:
+        left = np.arange(base, base + a)
+        right = np.arange(base + a, base + a + 3)
+        a_list.append(np.repeat(left, 3))
+        b_list.append(np.tile(right, a))
+        base += a + 3
+    # a sparse random background on the last 500 vertices
+    bg = base + rng.integers(0, 500, (2, 3000))
+    a_all = perm[np.concatenate(a_list + [bg[0]])]
+    b_all = perm[np.concatenate(b_list + [bg[1]])]
+    rp, col = SG._csr_from_pairs(n, a_all, b_all)
+    return SG.Graph(rp, col, dict(name="branches", sizes=sizes))
+
+
+@pytest.mark.timeout(900)
+def test_minhash_branch_edges_pass1_and_pass2(B):
+    """Rows of lengths 1..40,000 straddling every min-hash branch, in pass I
+    (the right vertices) and pass II (the left vertices' G_I groups), with
+    c1 = c2 = 40 (one 32-trial pass + an 8-trial tail pass split over
+    neighbour parts)."""
+    g = branch_graph()
+    deg = g.degrees()
+    for a in (1023, 1025, 2049, 16385, 40000):
+        assert (deg == a).sum() >= 3
+    out, ref = run_both(B, g, 2, 40, 21, 2, 40, 22, report=False)
+    assert_parity(out, ref, report=False)
+    sizes = np.diff(ref.G1.offs)[ref.s1p_group]
+    for a in (1024, 1025, 2048, 2049, 16384, 16385, 40000):
+        assert (sizes == a).any(), f"no pass-II row of {a} entries"
+
+
+@pytest.mark.parametrize("name", ["tiny", "small"])
+def test_grouping_v1_equals_v2(B, name, monkeypatch):
+    """The first grouping design (SG_GROUP_V1=1: two-level partition + warp
+    tier) and the second (one partition + shared-memory bucket sort) give
+    the same canonical G_I / G_II (both equal the oracle)."""
+    g = SG.make(name)
+    cfg = SG.CONFIGS[name]
+    args = (cfg["s1"], 33, cfg["seed1"], cfg["s2"], 35, cfg["seed2"])
+    out2, ref = run_both(B, g, *args, report=False)
+    assert_parity(out2, ref, report=False)
+    monkeypatch.setenv("SG_GROUP_V1", "1")
+    out1, _ = run_both(B, g, *args, report=False)
+    assert_parity(out1, ref, report=False)
 
 
 def test_edge_cases_empty_and_degenerate(B):
@@ -197,14 +268,18 @@ def test_trial_chunking_under_memory_budget(B, budget_mb, monkeypatch):
     assert abs(c["chunks1"]) > 1 or abs(c["chunks2"]) > 1, c
 
 
+@pytest.mark.parametrize("v1", [False, True])
 @pytest.mark.parametrize("target", ["4", "40", "300"])
-def test_two_level_partition_and_tiny_buckets(B, target, monkeypatch):
+def test_many_bins_and_tiny_buckets(B, target, v1, monkeypatch):
     """SG_GROUP_TARGET shrinks the target bucket size so that the small graph
-    takes the two-level partition (coarse scatter + per-bucket scatter) used by
-    the 40M-row trial segments of the GOS-shaped pass II."""
+    is partitioned into up to 2^13 bins per trial (two LSD digit passes in the
+    scatter, nearly empty buckets); with SG_GROUP_V1 the first design takes
+    its two-level partition."""
     g = SG.make("small")
     cfg = SG.CONFIGS["small"]
     monkeypatch.setenv("SG_GROUP_TARGET", target)
+    if v1:
+        monkeypatch.setenv("SG_GROUP_V1", "1")
     out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
                         report=False)
     assert_parity(out, ref, report=False)
@@ -302,6 +377,18 @@ def test_density_tiny_and_cliques(B):
         G.run(2, 50, 1, 2, 50, 2)
         labels, nc = G.report(0)
         assert nc == 3 and G.density(labels) == (1.0, 0.0, 3)
+        with pytest.raises(ValueError):                   # label array of the wrong length
+            G.density(labels[:-1])
+        with pytest.raises(ValueError):
+            G.agreement(labels, labels[:5])
+    # self-loops are not edges and one-directional entries count half (AMB-21)
+    for rp, col, lab in ((np.array([0, 2, 4], np.int64), np.array([0, 1, 0, 1], np.int32), [0, 0]),
+                         (np.array([0, 1, 3, 3], np.int64), np.array([1, 0, 2], np.int32), [0, 0, 0])):
+        lab = np.asarray(lab, np.int32)
+        with B.ShingleGraph(rp, col) as G:
+            got = G.density(lab)
+        want = oracle.cluster_density(rp, col, lab)
+        assert got[2] == want[2] and abs(got[0] - want[0]) <= 1e-12
 
 
 # ---------------------------------------------------------------- Eq. 2-5 pair counts
