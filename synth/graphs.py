@@ -96,15 +96,73 @@ def _pairs_within(rng, base, size, draws):
     return a, b
 
 
-def _unique(x):
-    """Sorted unique values (sort based; numpy's hash-based unique is slow here)."""
-    x = np.sort(x)
+def _unique(x, inplace=False):
+    """Sorted unique values (sort based; numpy's hash-based unique is slow here).
+    inplace=True sorts the caller's array in place (no copy)."""
+    if inplace:
+        x.sort()
+    else:
+        x = np.sort(x)
     if len(x) == 0:
         return x
     keep = np.empty(len(x), bool)
     keep[0] = True
     np.not_equal(x[1:], x[:-1], out=keep[1:])
     return x[keep]
+
+
+_BATCH = 1 << 25
+
+
+def _codes_within(rng, base, size, draws, n):
+    """Sorted unique undirected codes min*n + max of the pairs _pairs_within
+    would draw (same random stream: all first endpoints, then all second
+    endpoints), generated in batches so that memory stays O(draws) int32 +
+    the codes (the 640M-edge config)."""
+    draws = np.asarray(draws, np.int64)
+    tot = int(draws.sum())
+    if tot == 0:
+        return np.zeros(0, np.int64)
+    cum = np.cumsum(draws)
+    a = np.empty(tot, np.int32 if n < 2**31 else np.int64)
+    for s0 in range(0, tot, _BATCH):
+        e0 = min(tot, s0 + _BATCH)
+        blk = np.searchsorted(cum, np.arange(s0, e0, dtype=np.int64), side="right")
+        a[s0:e0] = base[blk] + np.floor(rng.random(e0 - s0) * size[blk]).astype(np.int64)
+    out = []
+    for s0 in range(0, tot, _BATCH):
+        e0 = min(tot, s0 + _BATCH)
+        blk = np.searchsorted(cum, np.arange(s0, e0, dtype=np.int64), side="right")
+        bb = base[blk] + np.floor(rng.random(e0 - s0) * size[blk]).astype(np.int64)
+        aa = a[s0:e0].astype(np.int64)
+        keep = aa != bb
+        aa, bb = aa[keep], bb[keep]
+        out.append(np.minimum(aa, bb) * n + np.maximum(aa, bb))
+    del a
+    codes = np.concatenate(out) if out else np.zeros(0, np.int64)
+    del out
+    return _unique(codes, inplace=True)
+
+
+def _csr_from_unique_codes(n, codes, perm):
+    """Simple symmetric CSR from sorted unique undirected codes lo*n + hi of
+    slots, relabelled by the permutation perm (a bijection, so the pairs stay
+    unique and loop-free): directed keys (src << 32 | dst), sorted in place."""
+    m = len(codes)
+    key = np.empty(2 * m, np.uint64)
+    for s0 in range(0, m, _BATCH):
+        e0 = min(m, s0 + _BATCH)
+        lo = perm[codes[s0:e0] // n].astype(np.uint64)
+        hi = perm[codes[s0:e0] % n].astype(np.uint64)
+        key[s0:e0] = (lo << np.uint64(32)) | hi
+        key[m + s0:m + e0] = (hi << np.uint64(32)) | lo
+    key.sort()
+    rows = key >> np.uint64(32)
+    row_ptr = np.zeros(n + 1, np.int64)
+    row_ptr[1:] = np.searchsorted(rows, np.arange(n, dtype=np.uint64), side="right")
+    del rows
+    col = np.ascontiguousarray(key.view(np.uint32)[0::2]).view(np.int32)
+    return row_ptr, col
 
 
 def _csr_from_pairs(n, a, b):
@@ -175,12 +233,10 @@ def homology_graph(n, n_isolated=0, m_target=None, seed=0,
         exp_link = max(budget - exp_fam_edges, 0.0)
     # sampling with replacement: -ln(1-d) * N draws give density ~ d
     draws = np.round(-np.log1p(-np.minimum(dens, 0.95)) * npairs).astype(np.int64)
-    a, b = _pairs_within(rng, fam_base, fam_sizes, draws)
-    ea.append(a)
-    eb.append(b)
     fixed = _codes(n, np.concatenate(ea[:n_cliques]) if n_cliques else np.zeros(0, np.int64),
                    np.concatenate(eb[:n_cliques]) if n_cliques else np.zeros(0, np.int64))
-    free = _codes(n, np.concatenate(ea[n_cliques:]), np.concatenate(eb[n_cliques:]))
+    del ea, eb
+    free = _codes_within(rng, fam_base, fam_sizes, draws, n)
     # linkers: random intra-component pairs, proportional to component size,
     # topped up until the undirected edge count reaches m_target (then trimmed)
     big = cc >= 3
@@ -191,12 +247,12 @@ def homology_graph(n, n_isolated=0, m_target=None, seed=0,
         if deficit <= 0 or not big.any():
             break
         ld = rng.poisson(2.0 * deficit * cc * big / max(int((cc * big).sum()), 1))
-        a, b = _pairs_within(rng, cc_base, cc, ld)
-        free = _unique(np.concatenate([free, _codes(n, a, b)]))
+        free = _unique(np.concatenate([free, _codes_within(rng, cc_base, cc, ld, n)]), inplace=True)
     excess = len(fixed) + len(free) - m_target
     if excess > 0:
         free = np.delete(free, rng.choice(len(free), excess, replace=False))
-    codes = _unique(np.concatenate([fixed, free]))
+    codes = free if len(fixed) == 0 else _unique(np.concatenate([fixed, free]), inplace=True)
+    del free
     # hubs (config 3): added on top of the m_target graph
     if n_hubs:
         non_iso = np.arange(n_isolated, n, dtype=np.int64)
@@ -207,9 +263,8 @@ def homology_graph(n, n_isolated=0, m_target=None, seed=0,
         hd = rng.integers(hub_lo, hub_hi + 1, n_hubs)
         codes = _unique(np.concatenate([codes, _codes(n, np.repeat(hubs, hd),
                                                      targets[rng.integers(0, len(targets), int(hd.sum()))])]))
-    lo = perm[codes // n]
-    hi = perm[codes % n]
-    row_ptr, col = _csr_from_pairs(n, lo, hi)
+    row_ptr, col = _csr_from_unique_codes(n, codes, perm)
+    del codes
     if not return_families:
         return row_ptr, col
     # planted partition (the "benchmark" of Eq. 2-5): cliques and families;
