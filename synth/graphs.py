@@ -27,8 +27,8 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-_DATA = os.environ.get("SG_DATA_DIR",
-                       os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "data"))
+# graph cache (outside the repo so it never travels with the gpurun snapshot)
+_DATA = os.environ.get("SG_DATA_DIR", "/tmp/sg_data")
 
 
 @dataclass

@@ -1,0 +1,79 @@
+"""Full-size bit-exact parity on the hub-heavy (BASELINE configs[2]) and the
+Pacific-Ocean-shaped 640M-edge (configs[3]) workloads, one GPU, against the
+digests the oracle's trial-outer run wrote (tools/oracle_digests.py ->
+tests/golden/digests_<config>.json): every pass-I column and every G_I trial,
+the S1' map, and listed pass-II columns / G_II trials, each read back trial by
+trial (sg_get_shingles_range / sg_get_groups_range).  The hub-heavy run also
+compares 200 sampled hub rows (degree > 10,000: block-per-vertex kernel,
+re-staged above 16,384 entries) with the oracle row by row."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import digests as D
+import oracle
+from synth import graphs as SG
+
+pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _gold(name):
+    p = os.path.join(GOLD, f"digests_{name}.json")
+    if not os.path.exists(p):
+        pytest.skip(f"no oracle digests for {name} (tools/oracle_digests.py {name})")
+    return json.load(open(p))
+
+
+@pytest.mark.timeout(3600)
+@pytest.mark.parametrize("name", ["hub2m", "pacific640m"])
+def test_fullsize_digests(name):
+    import torch
+    torch.cuda.init()
+    from paper_conf_ipps_wuk13_b200 import binding as B
+    gold = _gold(name)
+    cfg = SG.CONFIGS[name]
+    g = SG.make(name)
+    assert gold["graph_digest"] == D.column(np.concatenate([g.row_ptr.astype(np.uint64),
+                                                           g.col.astype(np.uint64)]))
+    h = B.shingle_graph_create(g.row_ptr, g.col)
+    try:
+        B.shingle_pass(h, cfg["s1"], cfg["c1"], cfg["seed1"])
+        B.group_by_shingle(h)
+        B.shingle_pass(h, cfg["s2"], cfg["c2"], cfg["seed2"])
+        B.group_by_shingle(h)
+        c = B.sg_get_counts(h)
+        for k in ("n_e", "groups1", "pairs1", "s1p", "entries2"):
+            assert c[k] == gold["counts"][k], k
+        rows1 = None
+        for j in range(cfg["c1"]):
+            m1, rows1 = B.sg_get_shingles_range(h, 1, j, j + 1)
+            assert D.column(np.ascontiguousarray(m1[:, 0])) == gold["dig_M1"][j], f"pass-I column {j}"
+            _, gid, offs, mem = B.sg_get_groups_range(h, 1, j, j + 1)
+            assert D.grouped_trial(gid, offs, mem) == gold["dig_G1"][j], f"G_I trial {j}"
+        assert D.column(rows1.astype(np.uint64)) == gold["rows1_digest"]
+        s1p, _ = B.sg_get_s1p(h)
+        assert D.column(s1p.astype(np.uint64)) == gold["s1p_digest"]
+        for i, t in enumerate(gold["keep2"]):
+            m2, _ = B.sg_get_shingles_range(h, 2, t, t + 1)
+            assert D.column(np.ascontiguousarray(m2[:, 0])) == gold["dig_M2k"][i], f"pass-II column {t}"
+            _, gid2, offs2, mem2 = B.sg_get_groups_range(h, 2, t, t + 1)
+            assert len(gid2) == gold["G2k_groups"][i]
+            assert D.grouped_trial(gid2, offs2, mem2) == gold["dig_G2k"][i], f"G_II trial {t}"
+        if name == "hub2m":
+            deg = g.degrees()
+            hubs = np.flatnonzero(deg > 10000)
+            assert len(hubs) >= 20000 and (deg > 16384).any()
+            A1, B1 = B.sg_get_hash_params(h, 1, cfg["c1"])
+            pick = np.random.default_rng(3).choice(hubs, 200, replace=False)
+            pick = np.union1d(pick, hubs[np.argsort(deg[hubs])[-5:]])        # the longest rows too
+            ids1, rows1 = B.sg_get_shingles(h, 1)
+            pos = np.searchsorted(rows1, pick)
+            for u, p in zip(pick, pos):
+                row = g.col[g.row_ptr[u]:g.row_ptr[u + 1]]
+                want = oracle.row_shingles(row, cfg["s1"], cfg["c1"], cfg["seed1"], A1, B1)
+                assert np.array_equal(ids1[p], want), f"hub row {u} (degree {deg[u]})"
+    finally:
+        B.shingle_graph_destroy(h)
