@@ -198,7 +198,7 @@ void free_pass(sg_graph *g, PassOut &p) {
   bool side = false;
   for (auto &ch : p.chunks) side |= ch.done != nullptr;
   if (side) cudaStreamSynchronize(g->side);       // chunks still in flight there
-  for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) dfree(g, *b);
+  for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid, &p.perm, &p.rstart_p, &p.rlen_p}) dfree(g, *b);
   for (auto &ch : p.chunks) {
     dfree(g, ch.keys);
     dfree(g, ch.ctr);
@@ -349,6 +349,41 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
   }
 }
 
+bool use_group_v1();
+
+// Pass II on one rank: lay the key positions out by row length so that rows
+// of <= 8 entries are processed one per lane (minhash_short_rows).  The
+// grouping is independent of the order of the pairs (v3 sorts each bucket by
+// (key, member)), and the value of key position i is perm[i] (the S1' index).
+void build_row_classes(sg_graph *g, PassOut &P, int64_t nrows) {
+  const int NC = short_row_max() + 2;
+  DBuf cnt, cur;
+  dalloc(g, cnt, (size_t)NC * 8);
+  dalloc(g, cur, (size_t)NC * 8);
+  CK(row_classes(ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), nrows, ptr<unsigned long long>(cnt),
+                 nullptr, nullptr, nullptr, nullptr, nullptr, g->stream));
+  std::vector<unsigned long long> h((size_t)NC);
+  CK(cudaMemcpyAsync(h.data(), cnt.p, (size_t)NC * 8, cudaMemcpyDeviceToHost, g->stream));
+  sync(g);
+  std::vector<unsigned long long> start((size_t)NC, 0);
+  unsigned long long run = 0;
+  for (int c = 0; c < NC; ++c) {
+    start[(size_t)c] = run;
+    run += h[(size_t)c];
+  }
+  const int64_t n_short = (int64_t)start[(size_t)NC - 1];   // rows of <= 8 entries
+  dalloc(g, P.perm, (size_t)nrows * 4);
+  dalloc(g, P.rstart_p, (size_t)nrows * 8);
+  dalloc(g, P.rlen_p, (size_t)nrows * 4);
+  CK(row_classes(ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), nrows, nullptr, ptr<unsigned long long>(cur),
+                 start.data(), ptr<uint32_t>(P.perm), ptr<int64_t>(P.rstart_p), ptr<int32_t>(P.rlen_p),
+                 g->stream));
+  sync(g);                                     // the host start table is read by the copy above
+  P.n_split = n_short / 16 * 16;
+  dfree(g, cnt);
+  dfree(g, cur);
+}
+
 // on_side: enqueue the kernels on the side stream after the buffers are
 // allocated in main-stream order; group_by_shingle waits on ch.done (the
 // chunk's keys and counters stay owned by the chunk until then).
@@ -367,8 +402,9 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_s
     st_begin(g, st_hash, st);
   }
   MinhashArgs a;
-  a.rstart = ptr<int64_t>(P.rstart);
-  a.rlen = ptr<int32_t>(P.rlen);
+  const bool perm = P.perm.p != nullptr;
+  a.rstart = ptr<int64_t>(perm ? P.rstart_p : P.rstart);
+  a.rlen = ptr<int32_t>(perm ? P.rlen_p : P.rlen);
   a.entries = P.entries;
   a.nrows = P.nrows;
   a.A = ptr<uint32_t>(P.A);
@@ -382,6 +418,16 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_s
   a.counter = ptr<unsigned long long>(ctr);
   a.hub_counter = a.counter + 1;
   a.tile_rows = st_hash == kStHash2 ? 16 : 8;   // pass II rows are short
+  if (perm && P.n_split > 0) {
+    // rows of <= 8 entries one per lane, then the rest with the tile kernels
+    MinhashArgs s = a;
+    s.nrows = P.n_split;
+    CK(minhash_short_rows(s, g->num_sms, st));
+    a.rstart += P.n_split;
+    a.rlen += P.n_split;
+    a.keys += P.n_split;                       // n_split % 16 == 0: tile stores stay aligned
+    a.nrows -= P.n_split;
+  }
   CK(minhash(a, g->num_sms, st));
   if (on_side) {
     st_end(g, st_hash, st);
@@ -412,7 +458,7 @@ bool use_group_v1();
 
 // Scratch bytes per pair of a trial segment of `maxseg` pairs (planning).
 double scratch_per_pair(int64_t maxseg) {
-  if (!use_group_v1()) return 12.5;          // v2: one partitioned copy (8 B key + 4 B value)
+  if (!use_group_v1()) return 12.5;          // v3: one partitioned copy (8 B key + 4 B value)
   int32_t b, b1;
   group_bits(maxseg, &b, &b1);
   return b == b1 ? 12.5 : 24.5;
@@ -587,27 +633,31 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
     npairs += L;
   }
   if (maxseg >= (int64_t)0xFFFFFFFFll) fail(g, SG_EOVERFLOW, "a trial segment exceeds 2^32 pairs");
-  int32_t bits = 0;
-  group_b_bits(maxseg, &bits);
-  const int64_t nbins = (int64_t)1 << bits;
+  int32_t bits1 = 0, fine = 0;
+  group_c_bits(maxseg, &bits1, &fine);
+  const int64_t nb = (int64_t)1 << bits1;
   GroupArgs a;
-  const int64_t nch = build_pieces(g, pieces, nt, S, a.plan, group_b_super_pairs());
+  build_pieces(g, pieces, nt, S, a.plan, group_c_chunk_pairs());
   std::vector<int64_t> seg((size_t)nt + 1);
   for (int j = 0; j <= nt; ++j) seg[(size_t)j] = seg_all[(size_t)t0 + j];
   upload(g, S.seg, seg.data(), seg.size() * 8);
-  need(g, S.counts, (size_t)(nch * nbins) * 4);
-  need(g, S.bstart1, (size_t)(nt * nbins) * 4);
-  need(g, S.bsize1, (size_t)(nt * nbins) * 4);
+  need(g, S.bstart1, (size_t)(nt * nb) * 4);
+  need(g, S.bsize1, (size_t)(nt * nb) * 4);
+  need(g, S.counts, (size_t)(nt * nb) * 4);          // the scatter's reservation cursors
   need(g, S.akeys, (size_t)npairs * 8);
   need(g, S.avals, (size_t)npairs * 4);
-  need(g, S.big_list, (size_t)(nt * nbins) * 4);
+  const int64_t scr = group_c_scratch_pairs(g->num_sms);
+  need(g, S.bkeys, (size_t)scr * 8);
+  need(g, S.bvals, (size_t)scr * 4);
+  need(g, S.big_list, (size_t)(nt * nb) * 4);
   need(g, S.big_count, 8);
   CK(cudaMemsetAsync(S.big_count.p, 0, 8, g->stream));
   a.plan.c = nt;
-  a.plan.bits = bits;
-  a.plan.bits1 = bits;
-  a.plan.nbins = nbins;
-  a.plan.nb1 = nbins;
+  a.plan.bits = bits1;
+  a.plan.bits1 = bits1;
+  a.plan.nbins = nb;
+  a.plan.nb1 = nb;
+  a.plan.fine_bits = fine;
   a.plan.npairs = npairs;
   a.plan.seg = ptr<int64_t>(S.seg);
   if (const char *lc = getenv("SG_LOCAL_CAP")) a.plan.local_cap = atoi(lc);   // test hook
@@ -615,27 +665,27 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
   a.vals = vals;
   a.rowid = rowid;
   a.val_base = val_base;
-  a.counts = ptr<uint32_t>(S.counts);
   a.bstart1 = a.bstart = ptr<uint32_t>(S.bstart1);
   a.bsize1 = a.bsize = ptr<uint32_t>(S.bsize1);
-  a.akeys = a.bkeys = ptr<uint64_t>(S.akeys);
-  a.avals = a.bvals = ptr<uint32_t>(S.avals);
+  a.gcur = ptr<uint32_t>(S.counts);
+  a.akeys = ptr<uint64_t>(S.akeys);
+  a.avals = ptr<uint32_t>(S.avals);
+  a.bkeys = ptr<uint64_t>(S.bkeys);
+  a.bvals = ptr<uint32_t>(S.bvals);
   a.big_list = ptr<uint32_t>(S.big_list);
   a.big_count = ptr<uint32_t>(S.big_count);
-  a.mid_list = nullptr;
-  a.mid_count = nullptr;
   a.members = ptr<uint32_t>(out.members);
   a.head = ptr<uint32_t>(out.head);
   a.okeys = okeys;
   st_begin(g, st_hist);
-  CK(group_b_hist(a, g->stream));
+  CK(group_c_hist(a, g->num_sms, g->stream));
   st_end(g, st_hist);
   st_begin(g, st_scatter);
-  CK(group_b_scatter(a, g->num_sms, g->stream));
+  CK(group_c_scatter(a, g->num_sms, g->stream));
   if (free_after_scatter) dfree(g, *free_after_scatter);   // keys consumed
   st_end(g, st_scatter);
   st_begin(g, st_local);
-  CK(group_b_local(a, g->num_sms, g->stream));
+  CK(group_c_bucket(a, g->num_sms, g->stream));
   st_end(g, st_local);
 }
 
@@ -1231,6 +1281,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
       CK(select_groups_write(ptr<uint32_t>(G1.head), G1.npairs, s, ptr<int64_t>(blk),
                              ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), g->stream));
       P.entries = ptr<uint32_t>(G1.members);
+      if (!g->xch && !use_group_v1() && nrows > 0) build_row_classes(g, P, nrows);
     }
     dfree(g, blk);
     dfree(g, tot);
@@ -1291,7 +1342,8 @@ sg_status group_by_shingle(sg_graph *g) {
       dalloc(g, out.members, (size_t)out.npairs * 4);
       dalloc(g, out.head, (size_t)((out.npairs + 31) / 32) * 4);
       CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
-      const uint32_t *rowid = level == 0 ? ptr<uint32_t>(P.rowid) : nullptr;
+      const uint32_t *rowid = level == 0 ? ptr<uint32_t>(P.rowid)
+                                         : (P.perm.p ? ptr<uint32_t>(P.perm) : nullptr);
       const uint32_t base = level == 0 ? 0u : (uint32_t)g->s1p_k0;
       GroupScratch S;
       for (auto &ch : P.chunks) {

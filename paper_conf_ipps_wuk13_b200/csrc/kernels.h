@@ -49,6 +49,17 @@ struct MinhashArgs {
 constexpr int kRowTile = 16;      // key_stride granule (multiple of every tile size)
 inline int64_t key_stride_for(int64_t nrows) { return (nrows + kRowTile - 1) / kRowTile * kRowTile; }
 cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st);
+// Rows of <= short_row_max() entries, one row per lane (pass II, DESIGN.md
+// §6.1): keys[j][r] for the a.nrows rows of (a.rstart, a.rlen).
+cudaError_t minhash_short_rows(const MinhashArgs &a, int num_sms, cudaStream_t st);
+int32_t short_row_max();
+// Length-class layout of rows: call with h_start == nullptr to count rows per
+// class (d_cnt[short_row_max() + 2] = rows of length 0..max, then longer),
+// then with the host class starts to write perm / rstart_p / rlen_p (classes
+// contiguous, ascending length, longer rows last; order inside a class free).
+cudaError_t row_classes(const int64_t *rstart, const int32_t *rlen, int64_t n, unsigned long long *d_cnt,
+                        unsigned long long *d_cursor, const unsigned long long *h_start, uint32_t *perm,
+                        int64_t *rstart_p, int32_t *rlen_p, cudaStream_t st);
 
 // Recompute shingle ids for (row, trial) requests (getters / report only).
 cudaError_t shingle_ids(const int64_t *rstart, const int32_t *rlen, const uint32_t *entries,
@@ -73,7 +84,8 @@ struct GroupPlan {
   int64_t *seg = nullptr;          // [c+1] output position of pair 0 of trial j (global)
   int32_t *trial_chunk0 = nullptr; // [c+1] first chunk of each trial
   int64_t chunk = 4096;            // pairs per chunk (the tables above)
-  int32_t local_cap = 0;           // grouping v2: largest bucket sorted in shared memory (0: default)
+  int32_t local_cap = 0;           // grouping v3: largest coarse bucket sorted by a CTA (0: default)
+  int32_t fine_bits = 0;           // grouping v3: fine (counting-sort) bits after the coarse bits
 };
 
 struct GroupArgs {
@@ -96,11 +108,56 @@ struct GroupArgs {
   uint32_t *big_count;         // [1] (zeroed by the caller)
   uint32_t *mid_list;          // [c*nbins] bucket ids with 1024 < size <= 4096 (CTA sort)
   uint32_t *mid_count;         // [1] (zeroed by the caller)
+  uint32_t *gcur = nullptr;    // v3: [c][nb1] running bucket reservation cursors
   // outputs
   uint32_t *members;           // [npairs]
   uint32_t *head;              // [(npairs+31)/32], zeroed by the launcher
   uint64_t *okeys = nullptr;   // [npairs] sorted keys (optional; multi-rank getters)
 };
+
+// ---- multi-rank helpers (kernels_pass.cu) ----------------------------------
+// counts[j] = number of rows whose rstart lies in [seg[j], seg[j+1]) (zeroed by caller)
+cudaError_t rows_per_trial(const int64_t *rstart, int64_t nrows, const int64_t *seg, int32_t c,
+                           unsigned long long *counts, cudaStream_t st);
+// rowid[i] = i + off[j] for the trial j with first[j] <= i < first[j+1]
+cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, const int64_t *off,
+                         int32_t c, cudaStream_t st);
+
+int64_t group_local_capacity();
+int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
+int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
+// Bucket plan for trial segments of at most `maxseg` pairs.
+void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
+// Fill plan.chunk_* (plan.nchunks entries) from the piece table (device
+// pointers; pieces ordered by trial, chunks of group_chunk_pairs() pairs).
+cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, const int64_t *p_in0,
+                               const int64_t *p_len, const int64_t *p_row0,
+                               const int64_t *p_chunk0, int32_t npieces, cudaStream_t st);
+cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
+cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st);   // chunk prefixes + bsize1 only
+cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
+cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level plans only
+// Sort every final bucket and write members + head bits: warp tier, then the
+// mid and big tiers over the lists the warp tier filled (no host sync).
+cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
+// Global-memory sort of the buckets listed in big_list (count on the device).
+cudaError_t group_big(const GroupArgs &g, int num_sms, cudaStream_t st);
+
+// ---- grouping v3 (kernels_sort.cu): coarse totals by the
+// top plan.bits1 (<= 11) key bits over chunks of group_c_chunk_pairs() pairs
+// (plan.chunk), an unordered coarse scatter with per-bucket atomic
+// reservations (gcur), then per coarse bucket a counting sort by the next
+// plan.fine_bits (<= 14) bits into a per-CTA scratch (bkeys / bvals,
+// group_c_scratch_pairs() pairs) and a (key, member) sort of every fine bucket.
+int64_t group_c_chunk_pairs();
+int32_t group_c_local_cap();
+int64_t group_c_scratch_pairs(int num_sms);
+void group_c_bits(int64_t maxseg, int32_t *bits1, int32_t *fine_bits);
+cudaError_t group_c_hist(const GroupArgs &g, int num_sms, cudaStream_t st);     // + bucket starts
+cudaError_t group_c_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
+cudaError_t group_c_bucket(const GroupArgs &g, int num_sms, cudaStream_t st);   // + big
+cudaError_t group_binscan(const GroupArgs &g, cudaStream_t st);   // bstart1 = scan of bsize1 per trial
 
 // ---- multi-rank helpers (kernels_pass.cu) ----------------------------------
 // counts[j] = number of rows whose rstart lies in [seg[j], seg[j+1]) (zeroed by caller)

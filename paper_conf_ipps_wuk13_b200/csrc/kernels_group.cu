@@ -470,6 +470,13 @@ cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+cudaError_t group_binscan(const GroupArgs &g, cudaStream_t st) {
+  if (g.plan.c == 0) return cudaSuccess;
+  binscan_kernel<<<(unsigned)g.plan.c, 1024, 0, st>>>(g);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
 cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
   cudaError_t e = group_colscan(g, st);
   if (e != cudaSuccess || g.plan.c == 0) return e;

@@ -517,6 +517,130 @@ cudaError_t launch_s(MhParams &P, int num_sms, cudaStream_t st) {
   return launch_tile<S, 8>(P, num_sms, st);
 }
 
+// ---- short rows, lane = row (pass II) ----------------------------------------
+// Pass-II rows are the member lists of first-level shingles: ~5 entries on
+// the GOS-shaped graph.  Rows of 2..8 entries are laid out by length class
+// (row_classes below) and taken 32 at a time by a warp, one row per lane: the
+// row sits in registers, every trial's (A, B) is a shared-memory broadcast,
+// and the 32 keys of a trial are one coalesced 256 B store.  A warp's rows
+// share their length except at the few class boundaries, so the predicated
+// 8-entry loop does not diverge.
+constexpr int kShortMax = 8;
+
+// One trial of a row held in registers: v[0, L) (L compile-time: no
+// predicated slots when the whole warp shares the length).
+template <int S, int L, bool PAD>
+__device__ __forceinline__ uint64_t row_key(const uint32_t (&v)[kShortMax], uint32_t A, uint32_t B,
+                                            uint64_t seed, int j) {
+  uint32_t m[S];
+#pragma unroll
+  for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+#pragma unroll
+  for (int e = 0; e < L; ++e) insert_min<S>(m, PAD ? hash_or_pad(A, B, v[e]) : m31_hash(A, B, v[e]));
+  return fmix(shingle_id<S>(m, seed, j));
+}
+
+template <int S, int L, bool PAD = false>
+__device__ __forceinline__ void rows_trials(const MinhashArgs &a, const uint32_t *sA, const uint32_t *sB,
+                                            const uint32_t (&v)[kShortMax], int64_t r, bool valid) {
+  uint64_t *dst = a.keys + r;
+  for (int j = 0; j < a.nt; ++j) {
+    const uint64_t key = row_key<S, L, PAD>(v, sA[j], sB[j], a.seed, a.t0 + j);
+    if (valid) dst[(int64_t)j * a.key_stride] = key;
+  }
+}
+
+template <int S>
+__global__ void __launch_bounds__(256) minhash_rows_kernel(const __grid_constant__ MinhashArgs a) {
+  extern __shared__ uint32_t sAB[];
+  uint32_t *sA = sAB, *sB = sAB + a.nt;
+  for (int i = threadIdx.x; i < a.nt; i += blockDim.x) {
+    sA[i] = a.A[a.t0 + i];
+    sB[i] = a.B[a.t0 + i];
+  }
+  __syncthreads();
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  for (int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w0 * 32 < a.nrows; w0 += nw) {
+    const int64_t r = w0 * 32 + lane;
+    const bool valid = r < a.nrows;
+    int len = 0;
+    uint32_t v[kShortMax];
+    if (valid) {
+      len = a.rlen[r];
+      const uint32_t *src = a.entries + a.rstart[r];
+#pragma unroll
+      for (int e = 0; e < kShortMax; ++e) v[e] = e < len ? src[e] : 0xFFFFFFFFu;
+    } else {
+#pragma unroll
+      for (int e = 0; e < kShortMax; ++e) v[e] = 0xFFFFFFFFu;
+    }
+    // rows are laid out by length class: the warp almost always shares one
+    // length (compile-time unrolled, no idle slots); at a class boundary the
+    // longest length is used, the padding (all-ones) never among the minima
+    const int lw = __reduce_max_sync(0xffffffffu, (unsigned)len);
+    const int lmin = __reduce_min_sync(0xffffffffu, (unsigned)len);
+    if (lmin != lw) {                          // class boundary / last rows: padded slots
+      rows_trials<S, kShortMax, true>(a, sA, sB, v, r, valid);
+      continue;
+    }
+    switch (lw) {
+      case 1: rows_trials<S, 1>(a, sA, sB, v, r, valid); break;
+      case 2: rows_trials<S, 2>(a, sA, sB, v, r, valid); break;
+      case 3: rows_trials<S, 3>(a, sA, sB, v, r, valid); break;
+      case 4: rows_trials<S, 4>(a, sA, sB, v, r, valid); break;
+      case 5: rows_trials<S, 5>(a, sA, sB, v, r, valid); break;
+      case 6: rows_trials<S, 6>(a, sA, sB, v, r, valid); break;
+      case 7: rows_trials<S, 7>(a, sA, sB, v, r, valid); break;
+      default: rows_trials<S, 8>(a, sA, sB, v, r, valid); break;
+    }
+  }
+}
+
+template <int S>
+cudaError_t launch_rows(const MinhashArgs &a, int num_sms, cudaStream_t st) {
+  const int64_t warps = (a.nrows + 31) / 32;
+  const int grid = (int)std::min<int64_t>((warps + 7) / 8, (int64_t)num_sms * 8);
+  minhash_rows_kernel<S><<<grid, 256, (size_t)a.nt * 8, st>>>(a);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+// ---- row classes: rows of 2..8 entries by length, then the longer ones --------
+__global__ void row_class_hist_kernel(const int32_t *__restrict__ rlen, int64_t n, unsigned long long *cnt) {
+  __shared__ unsigned int h[kShortMax + 2];
+  if (threadIdx.x < kShortMax + 2) h[threadIdx.x] = 0;
+  __syncthreads();
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&h[min(rlen[i], kShortMax + 1)], 1u);
+  __syncthreads();
+  if (threadIdx.x < kShortMax + 2 && h[threadIdx.x]) atomicAdd(&cnt[threadIdx.x], (unsigned long long)h[threadIdx.x]);
+}
+
+__global__ void row_class_scatter_kernel(const int64_t *__restrict__ rstart, const int32_t *__restrict__ rlen,
+                                         int64_t n, unsigned long long *cursor, uint32_t *perm,
+                                         int64_t *rstart_p, int32_t *rlen_p) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt = (1u << lane) - 1u;
+  for (int64_t i0 = ((int64_t)blockIdx.x * blockDim.x) & ~31ll; i0 < n; i0 += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = i0 + (threadIdx.x & ~31) + lane;
+    const bool valid = i < n;
+    const int len = valid ? rlen[i] : 0;
+    const int cls = valid ? min(len, kShortMax + 1) : -1;
+    const uint32_t peers = __match_any_sync(0xffffffffu, cls);
+    const int leader = __ffs(peers) - 1;
+    unsigned long long base = 0;
+    if (valid && lane == leader) base = atomicAdd(&cursor[cls], (unsigned long long)__popc(peers));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (valid) {
+      const int64_t p = (int64_t)base + __popc(peers & lt);
+      perm[p] = (uint32_t)i;
+      rstart_p[p] = rstart[i];
+      rlen_p[p] = len;
+    }
+  }
+}
+
 // ---- id recomputation for getters / report (one thread per request) --------
 __global__ void shingle_ids_kernel(const int64_t *rstart, const int32_t *rlen,
                                    const uint32_t *entries, const uint32_t *A, const uint32_t *B,
@@ -587,6 +711,42 @@ cudaError_t minhash(const MinhashArgs &a, int num_sms, cudaStream_t st) {
     case 8: return launch_s<8>(P, num_sms, st);
     default: return cudaErrorInvalidValue;
   }
+}
+
+cudaError_t minhash_short_rows(const MinhashArgs &a, int num_sms, cudaStream_t st) {
+  if (a.nrows == 0 || a.nt == 0) return cudaSuccess;
+  switch (a.s) {
+    case 1: return launch_rows<1>(a, num_sms, st);
+    case 2: return launch_rows<2>(a, num_sms, st);
+    case 3: return launch_rows<3>(a, num_sms, st);
+    case 4: return launch_rows<4>(a, num_sms, st);
+    case 5: return launch_rows<5>(a, num_sms, st);
+    case 6: return launch_rows<6>(a, num_sms, st);
+    case 7: return launch_rows<7>(a, num_sms, st);
+    case 8: return launch_rows<8>(a, num_sms, st);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+int32_t short_row_max() { return kShortMax; }
+
+cudaError_t row_classes(const int64_t *rstart, const int32_t *rlen, int64_t n, unsigned long long *d_cnt,
+                        unsigned long long *d_cursor, const unsigned long long *h_start, uint32_t *perm,
+                        int64_t *rstart_p, int32_t *rlen_p, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  if (!h_start) {
+    cudaError_t e = cudaMemsetAsync(d_cnt, 0, (kShortMax + 2) * 8, st);
+    if (e != cudaSuccess) return e;
+    row_class_hist_kernel<<<grid, 256, 0, st>>>(rlen, n, d_cnt);
+    ++g_launches;
+    return cudaGetLastError();
+  }
+  cudaError_t e = cudaMemcpyAsync(d_cursor, h_start, (kShortMax + 2) * 8, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return e;
+  row_class_scatter_kernel<<<grid, 256, 0, st>>>(rstart, rlen, n, d_cursor, perm, rstart_p, rlen_p);
+  ++g_launches;
+  return cudaGetLastError();
 }
 
 cudaError_t shingle_ids(const int64_t *rstart, const int32_t *rlen, const uint32_t *entries,

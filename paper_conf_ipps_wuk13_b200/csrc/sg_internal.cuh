@@ -100,6 +100,12 @@ struct PassOut {
   std::vector<KeyChunk> chunks; // trial chunks sized to the free HBM
   bool deferred = false;        // keys computed chunk by chunk inside group_by_shingle
   std::vector<int64_t> blocks;  // row blocks in generator order (multi-rank exchange pieces)
+  // pass II, one rank: key positions in length-class order;
+  // key position i belongs to row perm[i]; positions [0, n_split) are rows of
+  // <= 8 entries (one row per lane), the rest take the tile / hub kernels
+  DBuf perm;                    // uint32 [nrows] (empty: identity)
+  DBuf rstart_p, rlen_p;        // rstart / rlen in key-position order
+  int64_t n_split = 0;
 };
 
 // Grouped pairs of one level on this rank: per-trial segments of `members`
