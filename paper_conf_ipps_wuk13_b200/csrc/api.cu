@@ -444,13 +444,14 @@ struct GroupScratch {
   DBuf p_trial, p_in0, p_len, p_row0, p_chunk0, seg, trial_chunk0;
   DBuf chunk_i0, chunk_in0, chunk_len, chunk_trial;
   DBuf counts, bstart1, bsize1, bstart, bsize, akeys, avals, bkeys, bvals, big_list, big_count;
+  DBuf seg_pos, seg_len;
 };
 
 void free_scratch(sg_graph *g, GroupScratch &S) {
   for (DBuf *b : {&S.p_trial, &S.p_in0, &S.p_len, &S.p_row0, &S.p_chunk0, &S.seg, &S.trial_chunk0,
                   &S.chunk_i0, &S.chunk_in0, &S.chunk_len, &S.chunk_trial,
                   &S.counts, &S.bstart1, &S.bsize1, &S.bstart, &S.bsize, &S.akeys, &S.avals,
-                  &S.bkeys, &S.bvals, &S.big_list, &S.big_count})
+                  &S.bkeys, &S.bvals, &S.big_list, &S.big_count, &S.seg_pos, &S.seg_len})
     dfree(g, *b);
 }
 
@@ -458,7 +459,7 @@ bool use_group_v1();
 
 // Scratch bytes per pair of a trial segment of `maxseg` pairs (planning).
 double scratch_per_pair(int64_t maxseg) {
-  if (!use_group_v1()) return 12.5;          // v3: one partitioned copy (8 B key + 4 B value)
+  if (!use_group_v1()) return 13.9;          // v3: one partitioned copy (8 B key + 4 B value) + segment list
   int32_t b, b1;
   group_bits(maxseg, &b, &b1);
   return b == b1 ? 12.5 : 24.5;
@@ -650,8 +651,11 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
   need(g, S.bkeys, (size_t)scr * 8);
   need(g, S.bvals, (size_t)scr * 4);
   need(g, S.big_list, (size_t)(nt * nb) * 4);
-  need(g, S.big_count, 8);
-  CK(cudaMemsetAsync(S.big_count.p, 0, 8, g->stream));
+  need(g, S.big_count, 16);
+  CK(cudaMemsetAsync(S.big_count.p, 0, 16, g->stream));
+  const int64_t nseg = npairs / 9 + 1;                 // one-key fine buckets of >= 9 members
+  need(g, S.seg_pos, (size_t)nseg * 8);
+  need(g, S.seg_len, (size_t)nseg * 4);
   a.plan.c = nt;
   a.plan.bits = bits1;
   a.plan.bits1 = bits1;
@@ -674,6 +678,9 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
   a.bvals = ptr<uint32_t>(S.bvals);
   a.big_list = ptr<uint32_t>(S.big_list);
   a.big_count = ptr<uint32_t>(S.big_count);
+  a.seg_count = reinterpret_cast<unsigned long long *>(ptr<uint32_t>(S.big_count) + 2);
+  a.seg_pos = ptr<int64_t>(S.seg_pos);
+  a.seg_len = ptr<uint32_t>(S.seg_len);
   a.members = ptr<uint32_t>(out.members);
   a.head = ptr<uint32_t>(out.head);
   a.okeys = okeys;
@@ -686,6 +693,7 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
   st_end(g, st_scatter);
   st_begin(g, st_local);
   CK(group_c_bucket(a, g->num_sms, g->stream));
+  CK(group_c_segsort(a, g->num_sms, g->stream));
   st_end(g, st_local);
 }
 

@@ -109,6 +109,9 @@ struct GroupArgs {
   uint32_t *mid_list;          // [c*nbins] bucket ids with 1024 < size <= 4096 (CTA sort)
   uint32_t *mid_count;         // [1] (zeroed by the caller)
   uint32_t *gcur = nullptr;    // v3: [c][nb1] running bucket reservation cursors
+  unsigned long long *seg_count = nullptr;   // v3: one-key fine buckets of > 8 members left
+  int64_t *seg_pos = nullptr;                //   unsorted in `members`: output position,
+  uint32_t *seg_len = nullptr;               //   length (capacity npairs / 9 + 1)
   // outputs
   uint32_t *members;           // [npairs]
   uint32_t *head;              // [(npairs+31)/32], zeroed by the launcher
@@ -157,6 +160,8 @@ void group_c_bits(int64_t maxseg, int32_t *bits1, int32_t *fine_bits);
 cudaError_t group_c_hist(const GroupArgs &g, int num_sms, cudaStream_t st);     // + bucket starts
 cudaError_t group_c_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_c_bucket(const GroupArgs &g, int num_sms, cudaStream_t st);   // + big
+// Sort the members of every listed segment ascending (count read on the device).
+cudaError_t group_c_segsort(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_binscan(const GroupArgs &g, cudaStream_t st);   // bstart1 = scan of bsize1 per trial
 
 // ---- multi-rank helpers (kernels_pass.cu) ----------------------------------

@@ -44,9 +44,9 @@ using grp::bucket_extent;
 using grp::pair_less;
 
 constexpr int kHT = 1024;                 // histogram threads
-constexpr int kHPer = 8;                  // chunks per histogram CTA
-constexpr int kAT = 512;                  // scatter threads
-constexpr int kChunkA = 8192;             // pairs per chunk
+constexpr int kHPer = 16;                 // chunks per histogram CTA
+constexpr int kAT = 256;                  // scatter threads
+constexpr int kChunkA = 4096;             // pairs per chunk
 constexpr int kAPer = kChunkA / kAT;      // 16
 constexpr int kMaxB1 = 11;                // coarse bits
 constexpr int kMaxBins = 1 << kMaxB1;
@@ -56,10 +56,8 @@ constexpr int kMaxF = 14;                 // fine bits
 constexpr int kBCap = 65536;              // largest coarse bucket sorted by a CTA
 constexpr int kSmall = 8;                 // fine buckets sorted in registers
 constexpr int kWarpBuf = 256;             // fine buckets sorted by a warp
-constexpr int kMidMax = 4096;             // (unused)
-// fine buckets with 2.. pairs, listed per size class (region sizes per coarse bucket)
-constexpr int kL2 = 4096, kL4 = 2048, kL8 = 1024, kLW = 1024, kLM = 256;
-constexpr int kLTot = kL2 + kL4 + kL8 + kLW + kLM;
+// fine buckets with 2..8 pairs (sorted by a thread) and with more (a warp)
+constexpr int kL8 = 8192, kLW = 2048;
 constexpr int kBigMax = 64;               // CTA-sorted fine buckets listed per coarse bucket
 
 __device__ __forceinline__ uint32_t top_bits(uint64_t key, int B) {
@@ -133,12 +131,12 @@ struct ASmem {
   int64_t ws[33];
 };
 
-__global__ void __launch_bounds__(kAT, 2) scatter_c_kernel(const __grid_constant__ GroupArgs g) {
+__global__ void __launch_bounds__(kAT, 4) scatter_c_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   ASmem &S = *reinterpret_cast<ASmem *>(smraw);
   const int B = g.plan.bits1;
   const int nb = 1 << B;
-  constexpr int kBinsPer = kMaxBins / kAT;     // 4
+  constexpr int kBinsPer = kMaxBins / kAT;     // 8
   uint64_t kk[kAPer];
   auto load = [&](int64_t k) {
     const int64_t in0 = g.plan.chunk_in0[k];
@@ -212,29 +210,19 @@ __global__ void __launch_bounds__(kAT, 2) scatter_c_kernel(const __grid_constant
 }
 
 // ---- 3. per coarse bucket: counting sort by the fine bits + small sorts ----------
-constexpr int kBigSmem = 8192;            // fine buckets sorted by the CTA in shared memory
+constexpr int kBigSmem = 2048;            // multi-key fine buckets sorted by the CTA in shared memory
 
 struct BSmem {
   uint32_t cur[1 << kMaxF];              // fine counts -> starts -> ends
   uint32_t hb[kBCap / 32 + 2];           // head bits of the bucket
-  union {
-    struct {                             // per-warp sort buffers (9..256 pairs)
-      uint64_t k[kBW][kWarpBuf];
-      uint32_t v[kBW][kWarpBuf];
-    } w;
-    struct {                             // one CTA-wide sort (257..8192 pairs)
-      uint64_t k[kBigSmem];
-      uint32_t v[kBigSmem];
-    } c;
-  } buf;
-  uint32_t lst[kLTot];                   // fine buckets by size class: 2, 3-4, 5-8, 9-32, 33-256
+  uint64_t bk[kBigSmem];                 // one CTA-wide sort (rare: several keys, > 8 pairs)
+  uint32_t bv[kBigSmem];
+  uint32_t l8[kL8];                      // fine buckets of 2..8 pairs
+  uint32_t lw[kLW];                      // fine buckets of > 8 pairs
   uint32_t big[kBigMax];
-  uint32_t ncls[5], nbig;
+  uint32_t n8, nw, nbig;
   int64_t ws[33];
 };
-static_assert(sizeof(uint64_t) * kBW * kWarpBuf + sizeof(uint32_t) * kBW * kWarpBuf ==
-                  sizeof(uint64_t) * kBigSmem + sizeof(uint32_t) * kBigSmem,
-              "the two sort buffers share their storage");
 
 __device__ __forceinline__ void cswap(uint64_t &ka, uint32_t &va, uint64_t &kb, uint32_t &vb) {
   if (pair_less(kb, vb, ka, va)) {
@@ -284,8 +272,7 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
     const int64_t gbase = obase + sb;
     for (int i = threadIdx.x; i < nf; i += kBT) S.cur[i] = 0;
     for (int i = threadIdx.x; i < ((n + 31) >> 5) + 1; i += kBT) S.hb[i] = 0;
-    if (threadIdx.x < 5) S.ncls[threadIdx.x] = 0;
-    if (threadIdx.x == 0) S.nbig = 0;
+    if (threadIdx.x == 0) S.n8 = S.nw = S.nbig = 0;
     __syncthreads();
     // fine histogram
     {
@@ -356,24 +343,20 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
       const uint32_t hw = __ballot_sync(0xffffffffu, single);
       if (lane == 0 && hw) atomicOr(&S.hb[p >> 5], hw);
     }
-    // fine buckets of >= 2 pairs (a group, or keys sharing the fine bits):
-    // listed by size class, then sorted by (key, member) with every lane busy
+    // fine buckets of >= 2 pairs: almost always ONE group (one key) whose
+    // members only need ordering
     for (int f = threadIdx.x; f < nf; f += kBT) {
       const uint32_t e = S.cur[f];
       const uint32_t s = f ? S.cur[f - 1] : 0u;
       const uint32_t m = e - s;
       if (m <= 1) continue;
-      const int c = m == 2 ? 0 : m <= 4 ? 1 : m <= 8 ? 2 : m <= 32 ? 3 : m <= (uint32_t)kWarpBuf ? 4 : 5;
       bool listed = false;
-      if (c < 5) {
-        const int base = c == 0 ? 0 : c == 1 ? kL2 : c == 2 ? kL2 + kL4 : c == 3 ? kL2 + kL4 + kL8
-                                                                        : kL2 + kL4 + kL8 + kLW;
-        const int cap = c == 0 ? kL2 : c == 1 ? kL4 : c == 2 ? kL8 : c == 3 ? kLW : kLM;
-        const uint32_t t = atomicAdd(&S.ncls[c], 1u);
-        if (t < (uint32_t)cap) {
-          S.lst[base + t] = (uint32_t)f;
-          listed = true;
-        }
+      if (m <= kSmall) {
+        const uint32_t t = atomicAdd(&S.n8, 1u);
+        if (t < (uint32_t)kL8) { S.l8[t] = (uint32_t)f; listed = true; }
+      } else {
+        const uint32_t t = atomicAdd(&S.nw, 1u);
+        if (t < (uint32_t)kLW) { S.lw[t] = (uint32_t)f; listed = true; }
       }
       if (!listed) {
         const uint32_t u = atomicAdd(&S.nbig, 1u);
@@ -382,126 +365,81 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
     }
     __syncthreads();
     {
-      // 2 pairs: one compare-exchange
-      const int n2 = min(S.ncls[0], (uint32_t)kL2);
-      for (int x = threadIdx.x; x < n2; x += kBT) {
-        const int f = S.lst[x];
-        const uint32_t s = f ? S.cur[f - 1] : 0u;
-        uint64_t k0 = SK[s], k1 = SK[s + 1];
-        uint32_t v0 = SV[s], v1 = SV[s + 1];
-        cswap(k0, v0, k1, v1);
-        emit_one(g, S, gbase, s, k0, v0, true);
-        emit_one(g, S, gbase, s + 1, k1, v1, k1 != k0);
-      }
-      // 3-4 pairs: Batcher network on 4
-      const int n4 = min(S.ncls[1], (uint32_t)kL4);
-      for (int x = threadIdx.x; x < n4; x += kBT) {
-        const int f = S.lst[kL2 + x];
-        const uint32_t s = f ? S.cur[f - 1] : 0u;
-        const uint32_t m = S.cur[f] - s;
-        uint64_t k[4];
-        uint32_t v[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const bool in = (uint32_t)i < m;
-          k[i] = in ? SK[s + i] : ~0ull;
-          v[i] = in ? SV[s + i] : ~0u;
-        }
-        cswap(k[0], v[0], k[1], v[1]); cswap(k[2], v[2], k[3], v[3]);
-        cswap(k[0], v[0], k[2], v[2]); cswap(k[1], v[1], k[3], v[3]);
-        cswap(k[1], v[1], k[2], v[2]);
-#pragma unroll
-        for (int i = 0; i < 4; ++i)
-          if ((uint32_t)i < m) emit_one(g, S, gbase, s + i, k[i], v[i], i == 0 || k[i] != k[i - 1]);
-      }
-      // 5-8 pairs: Batcher odd-even merge network on 8 (pads sort last:
-      // members < 2^32 - 1)
-      const int n8 = min(S.ncls[2], (uint32_t)kL8);
+      // 2..8 pairs, one fine bucket per thread (every lane busy)
+      const int n8 = min(S.n8, (uint32_t)kL8);
       for (int x = threadIdx.x; x < n8; x += kBT) {
-        const int f = S.lst[kL2 + kL4 + x];
+        const int f = S.l8[x];
         const uint32_t s = f ? S.cur[f - 1] : 0u;
         const uint32_t m = S.cur[f] - s;
         uint64_t k[kSmall];
         uint32_t v[kSmall];
+        bool one = true;
 #pragma unroll
         for (int i = 0; i < kSmall; ++i) {
           const bool in = (uint32_t)i < m;
           k[i] = in ? SK[s + i] : ~0ull;
           v[i] = in ? SV[s + i] : ~0u;
+          one &= !in || k[i] == k[0];
         }
-        cswap(k[0], v[0], k[1], v[1]); cswap(k[2], v[2], k[3], v[3]);
-        cswap(k[4], v[4], k[5], v[5]); cswap(k[6], v[6], k[7], v[7]);
-        cswap(k[0], v[0], k[2], v[2]); cswap(k[1], v[1], k[3], v[3]);
-        cswap(k[4], v[4], k[6], v[6]); cswap(k[5], v[5], k[7], v[7]);
-        cswap(k[1], v[1], k[2], v[2]); cswap(k[5], v[5], k[6], v[6]);
-        cswap(k[0], v[0], k[4], v[4]); cswap(k[1], v[1], k[5], v[5]);
-        cswap(k[2], v[2], k[6], v[6]); cswap(k[3], v[3], k[7], v[7]);
-        cswap(k[2], v[2], k[4], v[4]); cswap(k[3], v[3], k[5], v[5]);
-        cswap(k[1], v[1], k[2], v[2]); cswap(k[3], v[3], k[4], v[4]);
-        cswap(k[5], v[5], k[6], v[6]);
+        if (one) {
+          // one group: order the members (pads ~0 sort last: members < 2^32 - 1)
+#define MS(a, b) { const uint32_t lo = min(v[a], v[b]); v[b] = max(v[a], v[b]); v[a] = lo; }
+          if (m == 2) {
+            MS(0, 1);
+          } else {
+            MS(0, 1); MS(2, 3); MS(4, 5); MS(6, 7); MS(0, 2); MS(1, 3); MS(4, 6); MS(5, 7);
+            MS(1, 2); MS(5, 6); MS(0, 4); MS(1, 5); MS(2, 6); MS(3, 7); MS(2, 4); MS(3, 5);
+            MS(1, 2); MS(3, 4); MS(5, 6);
+          }
+#undef MS
 #pragma unroll
-        for (int i = 0; i < kSmall; ++i)
-          if ((uint32_t)i < m) emit_one(g, S, gbase, s + i, k[i], v[i], i == 0 || k[i] != k[i - 1]);
+          for (int i = 0; i < kSmall; ++i)
+            if ((uint32_t)i < m) emit_one(g, S, gbase, s + i, k[0], v[i], i == 0);
+        } else {
+          // several keys share the fine bits: Batcher network on (key, member)
+          cswap(k[0], v[0], k[1], v[1]); cswap(k[2], v[2], k[3], v[3]);
+          cswap(k[4], v[4], k[5], v[5]); cswap(k[6], v[6], k[7], v[7]);
+          cswap(k[0], v[0], k[2], v[2]); cswap(k[1], v[1], k[3], v[3]);
+          cswap(k[4], v[4], k[6], v[6]); cswap(k[5], v[5], k[7], v[7]);
+          cswap(k[1], v[1], k[2], v[2]); cswap(k[5], v[5], k[6], v[6]);
+          cswap(k[0], v[0], k[4], v[4]); cswap(k[1], v[1], k[5], v[5]);
+          cswap(k[2], v[2], k[6], v[6]); cswap(k[3], v[3], k[7], v[7]);
+          cswap(k[2], v[2], k[4], v[4]); cswap(k[3], v[3], k[5], v[5]);
+          cswap(k[1], v[1], k[2], v[2]); cswap(k[3], v[3], k[4], v[4]);
+          cswap(k[5], v[5], k[6], v[6]);
+#pragma unroll
+          for (int i = 0; i < kSmall; ++i)
+            if ((uint32_t)i < m) emit_one(g, S, gbase, s + i, k[i], v[i], i == 0 || k[i] != k[i - 1]);
+        }
       }
-      // 9-32 pairs: a warp each, one pair per lane, bitonic by shuffles
-      const int nw32 = min(S.ncls[3], (uint32_t)kLW);
-      for (int x = w; x < nw32; x += kBW) {
-        const int f = S.lst[kL2 + kL4 + kL8 + x];
+      // > 8 pairs, a warp each: one key -> members written in place unsorted
+      // and the segment listed for the segmented member sort (group_c_segsort);
+      // several keys (rare) -> the CTA sort below
+      const int nwl = min(S.nw, (uint32_t)kLW);
+      for (int x = w; x < nwl; x += kBW) {
+        const int f = S.lw[x];
         const uint32_t s = f ? S.cur[f - 1] : 0u;
         const uint32_t m = S.cur[f] - s;
-        const bool in = (uint32_t)lane < m;
-        uint64_t k = in ? SK[s + lane] : ~0ull;
-        uint32_t v = in ? SV[s + lane] : ~0u;
-#pragma unroll
-        for (int kk = 2; kk <= 32; kk <<= 1)
-#pragma unroll
-          for (int jj = kk >> 1; jj > 0; jj >>= 1) {
-            const uint64_t ok = __shfl_xor_sync(0xffffffffu, k, jj);
-            const uint32_t ov = __shfl_xor_sync(0xffffffffu, v, jj);
-            const bool up = (lane & kk) == 0, lower = (lane & jj) == 0;
-            const bool other_less = pair_less(ok, ov, k, v);
-            if ((lower == up) ? other_less : !other_less) {
-              k = ok;
-              v = ov;
-            }
+        const uint64_t k0 = SK[s];
+        bool one = true;
+        for (uint32_t i = lane; i < m; i += 32) one &= SK[s + i] == k0;
+        one = __all_sync(0xffffffffu, one);
+        if (one) {
+          for (uint32_t i = lane; i < m; i += 32) {
+            g.members[gbase + s + i] = SV[s + i];
+            if (g.okeys) g.okeys[gbase + s + i] = k0;
           }
-        const uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
-        if (in) emit_one(g, S, gbase, s + lane, k, v, lane == 0 || prev != k);
-      }
-    }
-    // 33..256 pairs: a warp each, bitonic sort in its shared-memory buffer
-    const uint32_t nmid = min(S.ncls[4], (uint32_t)kLM);
-    for (uint32_t x = w; x < nmid; x += kBW) {
-      const int f = S.lst[kL2 + kL4 + kL8 + kLW + x];
-      const uint32_t e = S.cur[f];
-      const uint32_t s = f ? S.cur[f - 1] : 0u;
-      const int m = (int)(e - s);
-      int M = 64;
-      while (M < m) M <<= 1;
-      for (int i = lane; i < M; i += 32) {
-        S.buf.w.k[w][i] = i < m ? SK[s + i] : ~0ull;
-        S.buf.w.v[w][i] = i < m ? SV[s + i] : ~0u;
-      }
-      __syncwarp();
-      for (int kk = 2; kk <= M; kk <<= 1)
-        for (int jj = kk >> 1; jj > 0; jj >>= 1) {
-          for (int t = lane; t < (M >> 1); t += 32) {
-            const int a = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
-            const int b = (jj == (kk >> 1)) ? (a ^ (kk - 1)) : (a + jj);
-            uint64_t ka = S.buf.w.k[w][a], kb = S.buf.w.k[w][b];
-            uint32_t va = S.buf.w.v[w][a], vb = S.buf.w.v[w][b];
-            if (pair_less(kb, vb, ka, va)) {
-              S.buf.w.k[w][a] = kb;
-              S.buf.w.k[w][b] = ka;
-              S.buf.w.v[w][a] = vb;
-              S.buf.w.v[w][b] = va;
-            }
+          if (lane == 0) {
+            atomicOr(&S.hb[s >> 5], 1u << (s & 31));
+            const unsigned long long t = atomicAdd(g.seg_count, 1ull);
+            g.seg_pos[t] = gbase + s;
+            g.seg_len[t] = m;
           }
-          __syncwarp();
+        } else if (lane == 0) {
+          const uint32_t u = atomicAdd(&S.nbig, 1u);
+          if (u < kBigMax) S.big[u] = (uint32_t)f;
         }
-      for (int i = lane; i < m; i += 32)
-        emit_one(g, S, gbase, s + i, S.buf.w.k[w][i], S.buf.w.v[w][i], i == 0 || S.buf.w.k[w][i] != S.buf.w.k[w][i - 1]);
-      __syncwarp();
+      }
     }
     // larger fine buckets (a group of hundreds+ generators): the whole CTA,
     // bitonic in shared memory (<= 8192 pairs) or in the scratch; more than
@@ -524,8 +462,8 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
       const bool sm = M <= (uint32_t)kBigSmem;
       if (sm) {
         for (uint32_t i = threadIdx.x; i < M; i += kBT) {
-          S.buf.c.k[i] = i < m ? SK[s + i] : ~0ull;
-          S.buf.c.v[i] = i < m ? SV[s + i] : ~0u;
+          S.bk[i] = i < m ? SK[s + i] : ~0ull;
+          S.bv[i] = i < m ? SV[s + i] : ~0u;
         }
         __syncthreads();
       }
@@ -535,13 +473,13 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
             const uint32_t a = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
             const uint32_t b = (jj == (kk >> 1)) ? (a ^ (kk - 1)) : (a + jj);
             if (sm) {
-              const uint64_t ka = S.buf.c.k[a], kb = S.buf.c.k[b];
-              const uint32_t va = S.buf.c.v[a], vb = S.buf.c.v[b];
+              const uint64_t ka = S.bk[a], kb = S.bk[b];
+              const uint32_t va = S.bv[a], vb = S.bv[b];
               if (pair_less(kb, vb, ka, va)) {
-                S.buf.c.k[a] = kb;
-                S.buf.c.k[b] = ka;
-                S.buf.c.v[a] = vb;
-                S.buf.c.v[b] = va;
+                S.bk[a] = kb;
+                S.bk[b] = ka;
+                S.bv[a] = vb;
+                S.bv[b] = va;
               }
             } else if (b < m) {
               const uint64_t ka = SK[s + a], kb = SK[s + b];
@@ -557,9 +495,9 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
           __syncthreads();
         }
       for (uint32_t i = threadIdx.x; i < m; i += kBT) {
-        const uint64_t key = sm ? S.buf.c.k[i] : SK[s + i];
-        const uint64_t prev = i == 0 ? 0ull : (sm ? S.buf.c.k[i - 1] : SK[s + i - 1]);
-        emit_one(g, S, gbase, s + i, key, sm ? S.buf.c.v[i] : SV[s + i], i == 0 || prev != key);
+        const uint64_t key = sm ? S.bk[i] : SK[s + i];
+        const uint64_t prev = i == 0 ? 0ull : (sm ? S.bk[i - 1] : SK[s + i - 1]);
+        emit_one(g, S, gbase, s + i, key, sm ? S.bv[i] : SV[s + i], i == 0 || prev != key);
       }
       __syncthreads();
     }
@@ -584,6 +522,102 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
       }
     }
     __syncthreads();
+  }
+}
+
+// ---- 4. segmented member sort of one-key fine buckets of > 8 members --------
+constexpr int kSWT = 256;
+constexpr int kSWBuf = 1024;             // members per warp buffer
+constexpr int kSCBuf = 16384;            // members per CTA buffer
+
+__device__ __forceinline__ void bitonic32_u32(uint32_t &v, int lane) {
+#pragma unroll
+  for (int kk = 2; kk <= 32; kk <<= 1)
+#pragma unroll
+    for (int jj = kk >> 1; jj > 0; jj >>= 1) {
+      const uint32_t o = __shfl_xor_sync(0xffffffffu, v, jj);
+      const bool up = (lane & kk) == 0, lower = (lane & jj) == 0;
+      v = (lower == up) ? min(v, o) : max(v, o);
+    }
+}
+
+// bitonic sort of buf[0, M) (M a power of two) by nthr threads, index tid
+template <typename SYNC>
+__device__ __forceinline__ void bitonic_u32(uint32_t *buf, uint32_t M, uint32_t tid, uint32_t nthr,
+                                            SYNC sync) {
+  for (uint32_t kk = 2; kk <= M; kk <<= 1)
+    for (uint32_t jj = kk >> 1; jj > 0; jj >>= 1) {
+      for (uint32_t t = tid; t < (M >> 1); t += nthr) {
+        const uint32_t a = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
+        const uint32_t b = (jj == (kk >> 1)) ? (a ^ (kk - 1)) : (a + jj);
+        const uint32_t va = buf[a], vb = buf[b];
+        if (vb < va) {
+          buf[a] = vb;
+          buf[b] = va;
+        }
+      }
+      sync();
+    }
+}
+
+__global__ void __launch_bounds__(kSWT) segsort_warp_kernel(const __grid_constant__ GroupArgs g) {
+  __shared__ uint32_t buf[kSWT / 32][kSWBuf];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const unsigned long long n = *g.seg_count;
+  const unsigned long long nwarps = (unsigned long long)gridDim.x * (kSWT / 32);
+  for (unsigned long long x = (unsigned long long)blockIdx.x * (kSWT / 32) + w; x < n; x += nwarps) {
+    const uint32_t m = g.seg_len[x];
+    if (m > (uint32_t)kSWBuf) continue;
+    uint32_t *p = g.members + g.seg_pos[x];
+    if (m <= 32) {
+      uint32_t v = (uint32_t)lane < m ? p[lane] : ~0u;
+      bitonic32_u32(v, lane);
+      if ((uint32_t)lane < m) p[lane] = v;
+      continue;
+    }
+    uint32_t M = 64;
+    while (M < m) M <<= 1;
+    for (uint32_t i = lane; i < M; i += 32) buf[w][i] = i < m ? p[i] : ~0u;
+    __syncwarp();
+    bitonic_u32(buf[w], M, lane, 32, [] { __syncwarp(); });
+    for (uint32_t i = lane; i < m; i += 32) p[i] = buf[w][i];
+    __syncwarp();
+  }
+}
+
+__global__ void __launch_bounds__(1024) segsort_cta_kernel(const __grid_constant__ GroupArgs g) {
+  extern __shared__ uint32_t cbuf[];
+  const unsigned long long n = *g.seg_count;
+  for (unsigned long long x = blockIdx.x; x < n; x += gridDim.x) {
+    const uint32_t m = g.seg_len[x];
+    if (m <= (uint32_t)kSWBuf) continue;
+    uint32_t *p = g.members + g.seg_pos[x];
+    uint32_t M = 1;
+    while (M < m) M <<= 1;
+    if (M <= (uint32_t)kSCBuf) {
+      for (uint32_t i = threadIdx.x; i < M; i += blockDim.x) cbuf[i] = i < m ? p[i] : ~0u;
+      __syncthreads();
+      bitonic_u32(cbuf, M, threadIdx.x, blockDim.x, [] { __syncthreads(); });
+      for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) p[i] = cbuf[i];
+      __syncthreads();
+    } else {
+      // a group of more than 16K generators: in place in global memory
+      for (uint32_t kk = 2; kk <= M; kk <<= 1)
+        for (uint32_t jj = kk >> 1; jj > 0; jj >>= 1) {
+          for (uint32_t t = threadIdx.x; t < (M >> 1); t += blockDim.x) {
+            const uint32_t a = ((t & ~(jj - 1)) << 1) | (t & (jj - 1));
+            const uint32_t b = (jj == (kk >> 1)) ? (a ^ (kk - 1)) : (a + jj);
+            if (b < m) {
+              const uint32_t va = p[a], vb = p[b];
+              if (vb < va) {
+                p[a] = vb;
+                p[b] = va;
+              }
+            }
+          }
+          __syncthreads();
+        }
+    }
   }
 }
 
@@ -638,8 +672,24 @@ cudaError_t group_c_scatter(const GroupArgs &a, int num_sms, cudaStream_t st) {
   cudaError_t e = cudaFuncSetAttribute(scatter_c_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)smem);
   if (e != cudaSuccess) return e;
-  const int grid = (int)std::min<int64_t>((int64_t)num_sms * 2, a.plan.nchunks);
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, scatter_c_kernel, kAT, smem);
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * std::max(per_sm, 1), a.plan.nchunks);
   scatter_c_kernel<<<grid, kAT, smem, st>>>(a);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
+cudaError_t group_c_segsort(const GroupArgs &a, int num_sms, cudaStream_t st) {
+  segsort_warp_kernel<<<num_sms * 8, kSWT, 0, st>>>(a);
+  ++g_launches;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  const size_t smem = (size_t)kSCBuf * 4;
+  if ((e = cudaFuncSetAttribute(segsort_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)smem)) != cudaSuccess)
+    return e;
+  segsort_cta_kernel<<<num_sms, 1024, smem, st>>>(a);
   ++g_launches;
   return cudaGetLastError();
 }
