@@ -45,8 +45,8 @@ using grp::pair_less;
 
 constexpr int kHT = 1024;                 // histogram threads
 constexpr int kHPer = 16;                 // chunks per histogram CTA
-constexpr int kAT = 256;                  // scatter threads
-constexpr int kChunkA = 4096;             // pairs per chunk
+constexpr int kAT = 512;                  // scatter threads
+constexpr int kChunkA = 8192;             // pairs per chunk
 constexpr int kAPer = kChunkA / kAT;      // 16
 constexpr int kMaxB1 = 11;                // coarse bits
 constexpr int kMaxBins = 1 << kMaxB1;
@@ -58,7 +58,7 @@ constexpr int kSmall = 8;                 // fine buckets sorted in registers
 constexpr int kWarpBuf = 256;             // fine buckets sorted by a warp
 // fine buckets with 2..8 pairs (sorted by a thread) and with more (a warp)
 constexpr int kL8 = 8192, kLW = 2048;
-constexpr int kBigMax = 64;               // CTA-sorted fine buckets listed per coarse bucket
+constexpr int kBigMax = 256;              // CTA-sorted fine buckets listed per coarse bucket
 
 __device__ __forceinline__ uint32_t top_bits(uint64_t key, int B) {
   return B ? (uint32_t)(key >> (64 - B)) : 0u;
@@ -131,12 +131,12 @@ struct ASmem {
   int64_t ws[33];
 };
 
-__global__ void __launch_bounds__(kAT, 4) scatter_c_kernel(const __grid_constant__ GroupArgs g) {
+__global__ void __launch_bounds__(kAT, 2) scatter_c_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   ASmem &S = *reinterpret_cast<ASmem *>(smraw);
   const int B = g.plan.bits1;
   const int nb = 1 << B;
-  constexpr int kBinsPer = kMaxBins / kAT;     // 8
+  constexpr int kBinsPer = kMaxBins / kAT;     // 4
   uint64_t kk[kAPer];
   auto load = [&](int64_t k) {
     const int64_t in0 = g.plan.chunk_in0[k];
@@ -435,9 +435,64 @@ __global__ void __launch_bounds__(kBT, 1) bucket_c_kernel(const __grid_constant_
             g.seg_pos[t] = gbase + s;
             g.seg_len[t] = m;
           }
-        } else if (lane == 0) {
-          const uint32_t u = atomicAdd(&S.nbig, 1u);
-          if (u < kBigMax) S.big[u] = (uint32_t)f;
+        } else {
+          // several keys (a big group + keys sharing its fine bits): key runs in
+          // ascending key order, each run's members in place, then ordered
+          // (here when short, by the segmented sort when > 8)
+          const uint32_t lt = (1u << lane) - 1u;
+          uint32_t outp = s;
+          uint64_t last = 0;
+          bool first = true;
+          for (;;) {
+            uint64_t km = ~0ull;
+            bool any = false;
+            for (uint32_t i = lane; i < m; i += 32) {
+              const uint64_t kx = SK[s + i];
+              if ((first || kx > last) && kx <= km) {
+                km = kx;
+                any = true;
+              }
+            }
+            if (!__any_sync(0xffffffffu, any)) break;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+              const uint64_t ko = __shfl_xor_sync(0xffffffffu, km, o);
+              km = ko < km ? ko : km;
+            }
+            uint32_t cnt = 0;
+            for (uint32_t i0 = 0; i0 < m; i0 += 32) {
+              const uint32_t i = i0 + lane;
+              const bool sel = i < m && SK[s + i] == km;
+              const uint32_t mask = __ballot_sync(0xffffffffu, sel);
+              if (sel) {
+                const uint32_t pos = outp + cnt + __popc(mask & lt);
+                g.members[gbase + pos] = SV[s + i];
+                if (g.okeys) g.okeys[gbase + pos] = km;
+              }
+              cnt += __popc(mask);
+            }
+            __syncwarp();
+            if (lane == 0) {
+              atomicOr(&S.hb[outp >> 5], 1u << (outp & 31));
+              if (cnt > (uint32_t)kSmall) {
+                const unsigned long long t = atomicAdd(g.seg_count, 1ull);
+                g.seg_pos[t] = gbase + outp;
+                g.seg_len[t] = cnt;
+              } else {
+                uint32_t *p = g.members + gbase + outp;
+                for (uint32_t x = 1; x < cnt; ++x) {
+                  const uint32_t e = p[x];
+                  int y = (int)x - 1;
+                  while (y >= 0 && e < p[y]) { p[y + 1] = p[y]; --y; }
+                  p[y + 1] = e;
+                }
+              }
+            }
+            __syncwarp();
+            outp += cnt;
+            last = km;
+            first = false;
+          }
         }
       }
     }
@@ -644,12 +699,11 @@ void group_c_bits(int64_t maxseg, int32_t *bits1, int32_t *fine_bits) {
 
 cudaError_t group_c_hist(const GroupArgs &a, int num_sms, cudaStream_t st) {
   (void)num_sms;
-  if (a.plan.nchunks == 0) return cudaSuccess;
   const int B = a.plan.bits1;
   if (B < 0 || B > kMaxB1) return cudaErrorInvalidValue;
   const int64_t nb = (int64_t)1 << B;
   cudaError_t e = cudaMemsetAsync(a.bsize1, 0, (size_t)(a.plan.c * nb) * 4, st);
-  if (e != cudaSuccess) return e;
+  if (e != cudaSuccess || a.plan.nchunks == 0) return e;     // no pairs: every bucket empty
   const unsigned grid = (unsigned)((a.plan.nchunks + kHPer - 1) / kHPer);
   hist_c_kernel<<<grid, kHT, 0, st>>>(a);
   ++g_launches;
