@@ -616,11 +616,15 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   st_end(g, st_local);
 }
 
-// Grouping v2 (kernels_sort.cu): one stable partition by the
-// top B key bits over super-chunks, then one shared-memory sort per bucket.
-// Same contract as group_pieces.  SG_GROUP_V1=1 selects the first design
-// (A/B hook).
-bool use_group_v1() { return getenv("SG_GROUP_V1") != nullptr; }
+// Grouping design: the stable two-level partition + warp /
+// CTA local sorts (group_pieces, the default: measured fastest) or, with
+// SG_GROUP=v3, the order-independent design of kernels_sort.cu (coarse
+// atomic scatter + per-bucket counting sort + segmented member sort; parity-
+// green, measured slower; kept as the A/B alternative it was measured as).
+bool use_group_v1() {
+  const char *e = getenv("SG_GROUP");
+  return !(e && strcmp(e, "v3") == 0);
+}
 
 void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &pieces, int32_t t0,
                     int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,

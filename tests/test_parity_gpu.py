@@ -118,9 +118,10 @@ def test_big_bucket_path_large_clique(B):
 
 @pytest.mark.parametrize("cap", ["64", "1024"])
 def test_oversize_buckets_take_the_global_sort(B, cap, monkeypatch):
-    """SG_LOCAL_CAP shrinks the shared-memory bucket sort's capacity so that
-    buckets holding big groups (the 5,000-clique) and ordinary ones overflow
-    into the global-memory sort (big_kernel)."""
+    """SG_GROUP=v3 with SG_LOCAL_CAP shrinking the per-bucket sort's capacity
+    so that coarse buckets holding big groups (the 5,000-clique) and ordinary
+    ones overflow into the global-memory sort (big_kernel)."""
+    monkeypatch.setenv("SG_GROUP", "v3")
     monkeypatch.setenv("SG_LOCAL_CAP", cap)
     g = SG.cliques([5000, 300, 30, 12], n=6000, seed=4)
     out, ref = run_both(B, g, 2, 7, 13, 2, 6, 14)
@@ -173,15 +174,16 @@ def test_minhash_branch_edges_pass1_and_pass2(B):
 
 @pytest.mark.parametrize("name", ["tiny", "small"])
 def test_grouping_v1_equals_v2(B, name, monkeypatch):
-    """The first grouping design (SG_GROUP_V1=1: two-level partition + warp
-    tier) and the second (one partition + shared-memory bucket sort) give
-    the same canonical G_I / G_II (both equal the oracle)."""
+    """The default grouping (stable two-level partition + warp tier) and the
+    alternative SG_GROUP=v3 design (unordered coarse scatter + per-bucket
+    counting sort + segmented member sort, with pass-II rows in length-class
+    order) give the same canonical G_I / G_II (both equal the oracle)."""
     g = SG.make(name)
     cfg = SG.CONFIGS[name]
     args = (cfg["s1"], 33, cfg["seed1"], cfg["s2"], 35, cfg["seed2"])
     out2, ref = run_both(B, g, *args, report=False)
     assert_parity(out2, ref, report=False)
-    monkeypatch.setenv("SG_GROUP_V1", "1")
+    monkeypatch.setenv("SG_GROUP", "v3")
     out1, _ = run_both(B, g, *args, report=False)
     assert_parity(out1, ref, report=False)
 
@@ -268,18 +270,19 @@ def test_trial_chunking_under_memory_budget(B, budget_mb, monkeypatch):
     assert abs(c["chunks1"]) > 1 or abs(c["chunks2"]) > 1, c
 
 
-@pytest.mark.parametrize("v1", [False, True])
+@pytest.mark.parametrize("v3", [False, True])
 @pytest.mark.parametrize("target", ["4", "40", "300"])
-def test_many_bins_and_tiny_buckets(B, target, v1, monkeypatch):
+def test_many_bins_and_tiny_buckets(B, target, v3, monkeypatch):
     """SG_GROUP_TARGET shrinks the target bucket size so that the small graph
-    is partitioned into up to 2^13 bins per trial (two LSD digit passes in the
-    scatter, nearly empty buckets); with SG_GROUP_V1 the first design takes
-    its two-level partition."""
+    takes the two-level partition (coarse scatter + per-bucket scatter) used
+    by the 40M-row trial segments of the GOS-shaped pass II; with SG_GROUP=v3
+    the alternative design runs with up to 2^11 coarse bins and tiny
+    buckets."""
     g = SG.make("small")
     cfg = SG.CONFIGS["small"]
     monkeypatch.setenv("SG_GROUP_TARGET", target)
-    if v1:
-        monkeypatch.setenv("SG_GROUP_V1", "1")
+    if v3:
+        monkeypatch.setenv("SG_GROUP", "v3")
     out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
                         report=False)
     assert_parity(out, ref, report=False)
