@@ -170,26 +170,48 @@ __device__ __forceinline__ void emit_runs(const SplitSmem &S, int len, BIN bin_o
 }
 
 // ---- 1. histogram -----------------------------------------------------------
-__global__ void __launch_bounds__(kGThreads) hist_kernel(const __grid_constant__ GroupArgs g) {
-  __shared__ uint32_t hist[kMaxFan];
-  const int64_t nb = g.plan.nb1;
-  for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) hist[i] = 0;
-  __syncthreads();
-  const int64_t k = blockIdx.x;
-  const uint64_t *__restrict__ keys = g.keys + g.plan.chunk_in0[k];
-  const int len = g.plan.chunk_len[k];
-  uint64_t kk[kChunk / kGThreads];
+// kHistChunks consecutive chunks per 1024-thread CTA (long-running CTAs; the
+// next chunk's keys are loaded while the current one is counted).
+constexpr int kHThreads = 1024;
+constexpr int kHistChunks = 16;
+constexpr int kHPer = kChunk / kHThreads;      // 4 keys per thread per chunk
+
+__global__ void __launch_bounds__(kHThreads) hist_kernel(const __grid_constant__ GroupArgs g) {
+  __shared__ uint32_t hist[2][kMaxFan];
+  const int nb = (int)g.plan.nb1;
+  const int sh = pow2_shift(nb);
+  const int64_t k0 = (int64_t)blockIdx.x * kHistChunks;
+  const int64_t k1 = min(k0 + kHistChunks, g.plan.nchunks);
+  for (int i = threadIdx.x; i < 2 * kMaxFan; i += kHThreads) (&hist[0][0])[i] = 0;
+  uint64_t kk[kHPer], nx[kHPer];
+  auto load = [&](int64_t k, uint64_t (&dst)[kHPer]) {
+    const int len = g.plan.chunk_len[k];
+    const uint64_t *__restrict__ keys = g.keys + g.plan.chunk_in0[k];
 #pragma unroll
-  for (int u = 0; u < kChunk / kGThreads; ++u) {
-    const int i = threadIdx.x + u * kGThreads;
-    kk[u] = i < len ? keys[i] : 0;
+    for (int u = 0; u < kHPer; ++u) {
+      const int i = threadIdx.x + u * kHThreads;
+      dst[u] = i < len ? keys[i] : 0;
+    }
+  };
+  if (k0 < k1) load(k0, kk);
+  __syncthreads();
+  for (int64_t k = k0; k < k1; ++k) {
+    const int buf = (int)(k - k0) & 1;
+    if (k + 1 < k1) load(k + 1, nx);
+    const int len = g.plan.chunk_len[k];
+#pragma unroll
+    for (int u = 0; u < kHPer; ++u)
+      if (threadIdx.x + u * kHThreads < len)
+        atomicAdd(&hist[buf][sh >= 0 ? coarse_bin_pow2(kk[u], sh) : coarse_bin(kk[u], nb)], 1u);
+    __syncthreads();
+    uint32_t *out = g.counts + k * nb;
+    for (int i = threadIdx.x; i < nb; i += kHThreads) {
+      out[i] = hist[buf][i];
+      hist[buf][i] = 0;                       // ready for chunk k + 2
+    }
+#pragma unroll
+    for (int u = 0; u < kHPer; ++u) kk[u] = nx[u];
   }
-#pragma unroll
-  for (int u = 0; u < kChunk / kGThreads; ++u)
-    if (threadIdx.x + u * kGThreads < len) atomicAdd(&hist[coarse_bin(kk[u], nb)], 1u);
-  __syncthreads();
-  uint32_t *out = g.counts + k * nb;
-  for (int64_t i = threadIdx.x; i < nb; i += blockDim.x) out[i] = hist[i];
 }
 
 // ---- 2. offsets ---------------------------------------------------------------
@@ -457,7 +479,7 @@ cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, co
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
-  hist_kernel<<<(unsigned)g.plan.nchunks, kGThreads, 0, st>>>(g);
+  hist_kernel<<<(unsigned)((g.plan.nchunks + kHistChunks - 1) / kHistChunks), kHThreads, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
