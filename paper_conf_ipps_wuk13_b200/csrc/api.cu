@@ -215,22 +215,24 @@ void free_groups(sg_graph *g, Groups &q) {
 }
 
 // ---------------------------------------------------------------- validation
+// One warp per row (hub rows of tens of thousands of entries do not serialise
+// on one thread): row bounds, ids in [0, n), strictly increasing entries.
 __global__ void validate_kernel(const int64_t *rp, const int32_t *col, int64_t rows, int64_t nnz,
                                 int64_t n, int *bad) {
-  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < rows;
-       u += (int64_t)gridDim.x * blockDim.x) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; u < rows; u += nw) {
     const int64_t a = rp[u], b = rp[u + 1];
     if (b < a || a < 0 || b > nnz) {
-      atomicExch(bad, 1);
+      if (lane == 0) atomicExch(bad, 1);
       continue;
     }
-    for (int64_t e = a; e < b; ++e) {
+    bool ok = true;
+    for (int64_t e = a + lane; e < b; e += 32) {
       const int32_t v = col[e];
-      if (v < 0 || (int64_t)v >= n || (e > a && v <= col[e - 1])) {
-        atomicExch(bad, 1);
-        break;
-      }
+      ok &= v >= 0 && (int64_t)v < n && (e == a || v > col[e - 1]);
     }
+    if (!__all_sync(0xffffffffu, ok) && lane == 0) atomicExch(bad, 1);
   }
 }
 
@@ -1048,7 +1050,7 @@ void ingest(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr, const i
     DBuf bad;
     dalloc(g, bad, 4);
     CK(cudaMemsetAsync(bad.p, 0, 4, g->stream));
-    validate_kernel<<<std::min<int64_t>((rows + 255) / 256, 8192), 256, 0, g->stream>>>(
+    validate_kernel<<<std::min<int64_t>((rows + 7) / 8, (int64_t)g->num_sms * 16), 256, 0, g->stream>>>(
         ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col.p), rows,
         g->nnz_local, n, ptr<int>(bad));
     CK(cudaGetLastError());

@@ -111,6 +111,7 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
       pr[u] = __match_any_sync(vm, b);
       if ((pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
     }
+    __syncwarp();                      // the next batch's leaders read these counters
   }
   __syncthreads();
   {
