@@ -317,6 +317,32 @@ SG_API sg_status sg_s1p_offsets(int32_t world, int32_t rank, int32_t c1, const i
 SG_API sg_status sg_partition_rows(int64_t n, const int64_t *row_ptr, int32_t world, int64_t kappa,
                             int64_t *bounds);
 
+/* ------------------------------------------------------------------------ */
+/* Component sharding: pClust breaks the input graph into  */
+/* connected components before shingling.  Shingling only looks */
+/* at neighbourhoods, so no shingle, group or dense subgraph spans two       */
+/* components: whole components can be shingled on different GPUs with no    */
+/* exchange, every vertex taking its label from its own shard (the oracle's  */
+/* CC-locality self-check).  Pure host code (no GPU).                        */
+/*                                                                           */
+/* sg_component_shards: shard[n] <- the shard (0..world-1) of every vertex;  */
+/*   components (every stored entry an undirected edge) are placed heaviest  */
+/*   first on the least-loaded shard by sum(deg + kappa); load[world]        */
+/*   (optional) <- each shard's weight.  SG_EINVAL on a bad CSR.             */
+SG_API sg_status sg_component_shards(int64_t n, const int64_t *row_ptr, const int32_t *col,
+                                     int32_t world, int64_t kappa, int32_t *shard, int64_t *load);
+/* sg_shard_csr: the CSR of shard r over all n vertex ids (rows of the other */
+/*   shards empty): row_ptr_out[n+1], col_out[*nnz_out]; NULL outputs ->     */
+/*   only *nnz_out (two-call pattern).  Pass it to shingle_graph_create /    */
+/*   shingle_graph_load of the shard's GPU (world 1, no exchange).           */
+SG_API sg_status sg_shard_csr(int64_t n, const int64_t *row_ptr, const int32_t *col,
+                              const int32_t *shard, int32_t r, int64_t *row_ptr_out,
+                              int32_t *col_out, int64_t *nnz_out);
+/* sg_merge_shard_labels: out[v] = labels[shard[v] * n + v] (labels: the     */
+/*   world shards' report_dense_subgraphs labels stacked row by row).        */
+SG_API sg_status sg_merge_shard_labels(int64_t n, const int32_t *shard, int32_t world,
+                                       const int32_t *labels, int32_t *out);
+
 /* Library version / build string (sm_100a). */
 SG_API const char *sg_version(void);
 

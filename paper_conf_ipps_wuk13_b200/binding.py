@@ -83,6 +83,9 @@ def lib() -> C.CDLL:
         "sg_nccl_unique_id": (st, [vp]),
         "sg_s1p_offsets": (st, [i32, i32, i32, vp, vp, vp, vp]),
         "sg_version": (C.c_char_p, []),
+        "sg_component_shards": (st, [i64, vp, vp, i32, i64, vp, vp]),
+        "sg_shard_csr": (st, [i64, vp, vp, vp, i32, vp, vp, vp]),
+        "sg_merge_shard_labels": (st, [i64, vp, i32, vp, vp]),
     }
     for name, (rt, args) in sig.items():
         f = getattr(L, name)
@@ -345,6 +348,44 @@ def sg_s1p_offsets(all_counts, rank: int):
     _check(lib().sg_s1p_offsets(world, rank, c1, a.ctypes.data, first.ctypes.data, off.ctypes.data,
                                 C.byref(tot)))
     return first, off[:c1], tot.value
+
+
+def sg_component_shards(row_ptr, col, world: int, kappa: int = 8):
+    """Whole connected components per shard (N3): (shard int32[n], load int64[world])."""
+    row_ptr = np.ascontiguousarray(row_ptr, np.int64)
+    col = np.ascontiguousarray(col, np.int32)
+    n = len(row_ptr) - 1
+    shard = np.zeros(n, np.int32)
+    load = np.zeros(world, np.int64)
+    _check(lib().sg_component_shards(n, row_ptr.ctypes.data, col.ctypes.data, world, kappa,
+                                     shard.ctypes.data, load.ctypes.data))
+    return shard, load
+
+
+def sg_shard_csr(row_ptr, col, shard, r: int):
+    """CSR of shard r over all vertex ids (other rows empty)."""
+    row_ptr = np.ascontiguousarray(row_ptr, np.int64)
+    col = np.ascontiguousarray(col, np.int32)
+    shard = np.ascontiguousarray(shard, np.int32)
+    n = len(row_ptr) - 1
+    nnz = C.c_int64()
+    _check(lib().sg_shard_csr(n, row_ptr.ctypes.data, col.ctypes.data, shard.ctypes.data, r, None, None,
+                              C.byref(nnz)))
+    rp = np.zeros(n + 1, np.int64)
+    cl = np.zeros(nnz.value, np.int32)
+    _check(lib().sg_shard_csr(n, row_ptr.ctypes.data, col.ctypes.data, shard.ctypes.data, r,
+                              rp.ctypes.data, cl.ctypes.data, C.byref(nnz)))
+    return rp, cl
+
+
+def sg_merge_shard_labels(shard, labels_stacked):
+    """labels_stacked int32[world, n] (each shard's report) -> int32[n]."""
+    shard = np.ascontiguousarray(shard, np.int32)
+    lab = np.ascontiguousarray(labels_stacked, np.int32)
+    world, n = lab.shape
+    out = np.zeros(n, np.int32)
+    _check(lib().sg_merge_shard_labels(n, shard.ctypes.data, world, lab.ctypes.data, out.ctypes.data))
+    return out
 
 
 def sg_version() -> str:

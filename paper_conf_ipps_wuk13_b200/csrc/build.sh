@@ -6,7 +6,7 @@ cd "$(dirname "$0")"
 OUT=../libshingle.so
 NVCC=${NVCC:-/usr/local/cuda/bin/nvcc}
 FLAGS="-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v"
-SRCS="api.cu kernels_sort.cu kernels_pass.cu kernels_minhash.cu kernels_group.cu kernels_local.cu kernels_report.cu exchange.cu report.cpp"
+SRCS="api.cu kernels_sort.cu kernels_pass.cu kernels_minhash.cu kernels_group.cu kernels_local.cu kernels_report.cu exchange.cu report.cpp shards.cpp"
 OBJ=${SG_BUILD_DIR:-/tmp/sg_build_$$}
 mkdir -p "$OBJ"
 : > build.log
