@@ -14,6 +14,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "exchange.h"
 #include "kernels.h"
 #include "report.h"
@@ -149,7 +151,14 @@ int ev_take(sg_graph *g) {
   return (int)g->ev_next++;
 }
 
+// Stage names (NVTX ranges for a timeline profiler; sg_get_stage_ms order).
+const char *const kStageName[kNumStages] = {
+    "pass1", "group1", "pass2", "group2", "select1", "hash1", "select2", "hash2", "hist1",
+    "scatter1", "local1", "hist2", "scatter2", "local2", "exchange1", "exchange2", "fine1",
+    "fine2", "report"};
+
 void st_begin(sg_graph *g, int id, cudaStream_t st = nullptr) {
+  if (!st) nvtxRangePushA(kStageName[id]);     // host-side range (nested stages nest)
   const int e = ev_take(g);
   CK(cudaEventRecord(g->ev_pool[(size_t)e], st ? st : g->stream));
   g->st[id].push_back({e, -1});
@@ -159,6 +168,7 @@ void st_end(sg_graph *g, int id, cudaStream_t st = nullptr) {
   const int e = ev_take(g);
   CK(cudaEventRecord(g->ev_pool[(size_t)e], st ? st : g->stream));
   g->st[id].back().second = e;
+  if (!st) nvtxRangePop();
 }
 
 void st_clear(sg_graph *g) {
