@@ -49,6 +49,11 @@ typedef struct sg_graph sg_graph;
 /* create() flags */
 #define SG_DEVICE_PTRS 0x1u   /* row_ptr / col are device pointers (on dist->device) */
 #define SG_NO_VALIDATE 0x2u   /* skip the CSR validation (caller guarantees it)   */
+#define SG_HOST_CSR    0x4u   /* out-of-core entries: col stays in host memory, page-locked */
+                              /* and mapped (cudaHostRegister), and the kernels read it over */
+                              /* the host link; only row_ptr is copied to HBM.  The caller  */
+                              /* keeps `col` alive and unchanged until the handle is         */
+                              /* destroyed or re-loaded.                   */
 #define SG_REPORT_HOST 0x10   /* report_dense_subgraphs mode flag: host union-find */
 
 /* Multi-GPU description: one process (or, with loopback, one host thread) per

@@ -20,6 +20,7 @@ LIB_PATH = os.environ.get("SG_LIB") or os.path.join(_HERE, "libshingle.so")
 SG_OK, SG_EINVAL, SG_ENOMEM, SG_ESTATE, SG_ECUDA, SG_ENCCL, SG_EOVERFLOW = range(7)
 SG_DEVICE_PTRS = 0x1
 SG_NO_VALIDATE = 0x2
+SG_HOST_CSR = 0x4
 STATUS_NAMES = {0: "SG_OK", 1: "SG_EINVAL", 2: "SG_ENOMEM", 3: "SG_ESTATE", 4: "SG_ECUDA",
                 5: "SG_ENCCL", 6: "SG_EOVERFLOW"}
 STAGES = ["pass1", "group1", "pass2", "group2", "select1", "hash1", "select2", "hash2",
@@ -113,15 +114,19 @@ def _is_cuda(x) -> bool:
 
 
 # ------------------------------------------------------------------ C ABI calls
-def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dict] = None):
-    """row_ptr int64[n+1], col int32[nnz]: numpy arrays (host) or CUDA tensors."""
+def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dict] = None,
+                         host_csr: bool = False):
+    """row_ptr int64[n+1], col int32[nnz]: numpy arrays (host) or CUDA tensors.
+    host_csr: out-of-core entries (col stays in host memory, mapped; keep the
+    array alive and unchanged while the handle uses it)."""
     dev = _is_cuda(row_ptr)
     if not dev:
         row_ptr = np.ascontiguousarray(row_ptr, np.int64)
         col = np.ascontiguousarray(col, np.int32)
     n = int(row_ptr.shape[0]) - 1
     nnz = int(col.shape[0])
-    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE)
+    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE) | \
+        (SG_HOST_CSR if host_csr else 0)
     dptr = None
     if dist is not None:
         d = sg_dist(int(dist.get("rank", 0)), int(dist.get("world", 1)), int(dist.get("device", 0)),
@@ -138,14 +143,15 @@ def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dic
     return out
 
 
-def shingle_graph_load(h, row_ptr, col, validate: bool = True):
+def shingle_graph_load(h, row_ptr, col, validate: bool = True, host_csr: bool = False):
     """Replace the resident graph of handle h (host arrays or CUDA tensors)."""
     dev = _is_cuda(row_ptr)
     if not dev:
         row_ptr = np.ascontiguousarray(row_ptr, np.int64)
         col = np.ascontiguousarray(col, np.int32)
     n = int(row_ptr.shape[0]) - 1
-    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE)
+    flags = (SG_DEVICE_PTRS if dev else 0) | (0 if validate else SG_NO_VALIDATE) | \
+        (SG_HOST_CSR if host_csr else 0)
     _check(lib().shingle_graph_load(h, n, int(col.shape[0]), _addr(row_ptr), _addr(col), flags), h)
 
 
@@ -396,8 +402,9 @@ def sg_version() -> str:
 class ShingleGraph:
     """RAII wrapper: create -> pass -> group -> pass -> group -> report."""
 
-    def __init__(self, row_ptr, col, validate=True, dist=None):
-        self.h = shingle_graph_create(row_ptr, col, validate=validate, dist=dist)
+    def __init__(self, row_ptr, col, validate=True, dist=None, host_csr=False):
+        self._keep = (row_ptr, col) if host_csr else None      # mapped by the handle
+        self.h = shingle_graph_create(row_ptr, col, validate=validate, dist=dist, host_csr=host_csr)
         self.n = int(row_ptr.shape[0]) - 1
 
     def run(self, s1, c1, seed1, s2, c2, seed2):

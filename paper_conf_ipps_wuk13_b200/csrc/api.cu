@@ -1025,8 +1025,15 @@ void host_groups(sg_graph *g, int level, HostGroups &H, bool want_ids, int t0 = 
 
 // Copy this rank's row range of a host (or device) CSR into HBM, rebase it
 // and validate it on the device (create and load).
+void unmap_col(sg_graph *g) {
+  if (g->col_reg) cudaHostUnregister(g->col_reg);
+  cudaGetLastError();
+  g->col_reg = nullptr;
+  g->col_dev = nullptr;
+}
+
 void ingest(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr, const int64_t *rp_host,
-            const int32_t *col, bool devptr, bool validate) {
+            const int32_t *col, bool devptr, bool validate, bool host_csr = false) {
   g->n = n;
   g->nnz_global = nnz;
   // row range of this rank
@@ -1043,11 +1050,36 @@ void ingest(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr, const i
   if (e0 < 0 || e1 < e0 || e1 > nnz) fail(g, SG_EINVAL, "invalid CSR: row_ptr is not monotone within [0, nnz]");
   g->nnz_local = e1 - e0;
   dalloc(g, g->row_ptr, (size_t)(rows + 1) * 8);
-  dalloc(g, g->col, (size_t)g->nnz_local * 4);
+  unmap_col(g);
+  const bool mapped = host_csr && !devptr;
+  if (mapped) {
+    // out-of-core entries: page-lock and map the caller's slice; the kernels
+    // read it over the host link (N4)
+    dfree(g, g->col);
+    if (g->nnz_local) {
+      void *h = const_cast<int32_t *>(col + e0);
+      cudaError_t e = cudaHostRegister(h, (size_t)g->nnz_local * 4,
+                                       cudaHostRegisterMapped | cudaHostRegisterReadOnly);
+      if (e == cudaErrorHostMemoryAlreadyRegistered) cudaGetLastError();   // the caller pinned it
+      else {
+        CK(e);
+        g->col_reg = h;
+      }
+      void *d = nullptr;
+      CK(cudaHostGetDevicePointer(&d, h, 0));
+      g->col_dev = reinterpret_cast<const uint32_t *>(d);
+    } else {
+      dalloc(g, g->col, 16);
+      g->col_dev = ptr<uint32_t>(g->col);
+    }
+  } else {
+    dalloc(g, g->col, (size_t)g->nnz_local * 4);
+    g->col_dev = ptr<uint32_t>(g->col);
+  }
   const cudaMemcpyKind kind = devptr ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
   if (n > 0) {
     CK(cudaMemcpyAsync(g->row_ptr.p, row_ptr + g->row_lo, (rows + 1) * 8, kind, g->stream));
-    if (g->nnz_local)
+    if (g->nnz_local && !mapped)
       CK(cudaMemcpyAsync(g->col.p, col + e0, g->nnz_local * 4, kind, g->stream));
     rebase_kernel<<<std::min<int64_t>((rows + 256) / 256, 4096), 256, 0, g->stream>>>(
         ptr<int64_t>(g->row_ptr), rows + 1, e0);
@@ -1061,7 +1093,7 @@ void ingest(sg_graph *g, int64_t n, int64_t nnz, const int64_t *row_ptr, const i
     dalloc(g, bad, 4);
     CK(cudaMemsetAsync(bad.p, 0, 4, g->stream));
     validate_kernel<<<std::min<int64_t>((rows + 7) / 8, (int64_t)g->num_sms * 16), 256, 0, g->stream>>>(
-        ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col.p), rows,
+        ptr<int64_t>(g->row_ptr), reinterpret_cast<const int32_t *>(g->col_dev), rows,
         g->nnz_local, n, ptr<int>(bad));
     CK(cudaGetLastError());
     int hb = 0;
@@ -1190,7 +1222,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
     CK(cudaMemPoolCreate(&g->pool, &pp));
     uint64_t thr = UINT64_MAX;
     CK(cudaMemPoolSetAttribute(g->pool, cudaMemPoolAttrReleaseThreshold, &thr));
-    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, validate);
+    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, validate, (flags & SG_HOST_CSR) != 0);
     if (g->world > 1 || (dist && (dist->flags & SG_DIST_EXCHANGE))) g->xch = exchange_create(g, dist);
     sync(g);
     g->launch_base = g_launches.load();
@@ -1208,6 +1240,7 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
       cudaStreamSynchronize(g->stream);
     }
     cudaGetLastError();
+    unmap_col(g);
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
     if (g->side) cudaStreamDestroy(g->side);
     if (g->pool) cudaMemPoolDestroy(g->pool);
@@ -1242,7 +1275,8 @@ sg_status shingle_graph_load(sg_graph *g, int64_t n, int64_t nnz, const int64_t 
     g->e2_global = -1;
     g->ov_valid = false;
     g->state = kEmpty;                  // until the new graph is resident and valid
-    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, !(flags & SG_NO_VALIDATE));
+    ingest(g, n, nnz, row_ptr, rp_host, col, devptr, !(flags & SG_NO_VALIDATE),
+           (flags & SG_HOST_CSR) != 0);
     sync(g);
     g->state = kCreated;
     g->launch_base = g_launches.load();
@@ -1291,7 +1325,7 @@ sg_status shingle_pass(sg_graph *g, int32_t s, int32_t c, uint64_t seed) {
       CK(select_csr_write(ptr<int64_t>(g->row_ptr), rows, s, g->row_lo, ptr<int64_t>(blk),
                           ptr<int64_t>(P.rstart), ptr<int32_t>(P.rlen), ptr<uint32_t>(P.rowid),
                           g->stream));
-      P.entries = ptr<uint32_t>(g->col);
+      P.entries = g->col_dev;
     } else {
       Groups &G1 = g->grp[0];
       dalloc(g, blk, (size_t)sel_scratch_elems((G1.npairs + 31) / 32) * 8);
@@ -1438,6 +1472,7 @@ void shingle_graph_destroy(sg_graph *g) {
     for (auto &ch : g->pass[l].chunks)
       if (ch.done) cudaEventDestroy(ch.done);
   if (g->xch) exchange_destroy(g->xch);
+  unmap_col(g);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   if (g->side) cudaStreamDestroy(g->side);
   if (g->pool) cudaMemPoolDestroy(g->pool);
@@ -1652,7 +1687,7 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
       a.A2 = ptr<uint32_t>(P2.A);
       a.B2 = ptr<uint32_t>(P2.B);
       a.row_ptr = ptr<int64_t>(g->row_ptr);
-      a.col = ptr<uint32_t>(g->col);
+      a.col = g->col_dev;
       a.members1 = ptr<uint32_t>(g->grp[0].members);
       a.rows1 = P1.nrows;
       a.rstart2 = ptr<int64_t>(P2.rstart);
@@ -1716,7 +1751,11 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
     std::vector<int32_t> hcol;
     if (P1.s >= 3 && mode == 0) {
       hrp = d2h<int64_t>(g, g->row_ptr, (size_t)(g->row_hi - g->row_lo + 1));
-      hcol = d2h<int32_t>(g, g->col, (size_t)g->nnz_local);
+      hcol.resize((size_t)g->nnz_local);
+      if (g->nnz_local) {
+        CK(cudaMemcpyAsync(hcol.data(), g->col_dev, (size_t)g->nnz_local * 4, cudaMemcpyDefault, g->stream));
+        sync(g);
+      }
     }
     ReportInput in;
     in.n = g->n;
@@ -1755,7 +1794,7 @@ static void overlap_compute(sg_graph *g, int32_t mode, int32_t min_size) {
     a.A1 = ptr<uint32_t>(P1.A);
     a.B1 = ptr<uint32_t>(P1.B);
     a.row_ptr = ptr<int64_t>(g->row_ptr);
-    a.col = ptr<uint32_t>(g->col);
+    a.col = g->col_dev;
     a.members1 = ptr<uint32_t>(g->grp[0].members);
     a.rows1 = P1.nrows;
     a.rstart2 = ptr<int64_t>(P2.rstart);
@@ -1851,7 +1890,7 @@ sg_status sg_cluster_density(sg_graph *g, const int32_t *labels, int32_t min_siz
     dalloc(g, de, (size_t)n * 8);
     dalloc(g, ds, (size_t)n * 4);
     CK(cudaMemcpyAsync(dl.p, labels, (size_t)n * 4, cudaMemcpyHostToDevice, g->stream));
-    CK(density_device(ptr<int64_t>(g->row_ptr), ptr<uint32_t>(g->col), n, ptr<int32_t>(dl),
+    CK(density_device(ptr<int64_t>(g->row_ptr), g->col_dev, n, ptr<int32_t>(dl),
                       ptr<unsigned long long>(de), ptr<uint32_t>(ds), g->num_sms, g->stream));
     std::vector<unsigned long long> e2((size_t)n);
     std::vector<uint32_t> sz((size_t)n);
@@ -1928,7 +1967,7 @@ sg_status sg_connected_components(sg_graph *g, int32_t *labels, int64_t *n_compo
     DBuf parent, dl;
     dalloc(g, parent, (size_t)n * 4);
     dalloc(g, dl, (size_t)n * 4);
-    CK(components_device(ptr<int64_t>(g->row_ptr), ptr<uint32_t>(g->col), n,
+    CK(components_device(ptr<int64_t>(g->row_ptr), g->col_dev, n,
                          ptr<uint32_t>(parent), ptr<int32_t>(dl), g->num_sms, g->stream));
     if (n) CK(cudaMemcpyAsync(labels, dl.p, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
     sync(g);

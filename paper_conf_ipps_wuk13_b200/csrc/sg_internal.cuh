@@ -158,7 +158,10 @@ struct sg_graph {
   int64_t row_lo = 0, row_hi = 0;
   int64_t nnz_local = 0;
   sg::DBuf row_ptr;   // int64 [rows + 1], rebased to 0
-  sg::DBuf col;       // uint32 [nnz_local]
+  sg::DBuf col;       // uint32 [nnz_local] (empty with SG_HOST_CSR)
+  const uint32_t *col_dev = nullptr;   // the entries as the kernels read them: col.p, or the
+                                       // device alias of the caller's mapped host array
+  void *col_reg = nullptr;             // host range this handle registered (SG_HOST_CSR)
   // passes and groups
   sg::PassOut pass[2];
   sg::Groups grp[2];

@@ -441,3 +441,30 @@ def test_components(B, name):
         lab, k = G.components()
     want, wk = oracle.connected_components(g.row_ptr, g.col)
     assert k == wk and np.array_equal(lab, want)
+
+
+@pytest.mark.parametrize("name", ["tiny", "hubsmall"])
+def test_out_of_core_entries_host_csr(B, name):
+    """SG_HOST_CSR (N4): the entries stay in host memory (page-locked, mapped)
+    and the kernels read them over the host link; every output, the reports,
+    density and components equal the oracle / the in-HBM run."""
+    g = SG.make(name)
+    cfg = SG.CONFIGS[name]
+    args = (cfg["s1"], 40, cfg["seed1"], cfg["s2"], 33, cfg["seed2"])
+    col = np.ascontiguousarray(g.col)
+    with B.ShingleGraph(g.row_ptr, col, host_csr=True) as G:
+        G.run(*args)
+        out = dict(
+            M1=B.sg_get_shingles(G.h, 1), G1=B.sg_get_groups(G.h, 1), s1p=B.sg_get_s1p(G.h),
+            M2=B.sg_get_shingles(G.h, 2), G2=B.sg_get_groups(G.h, 2), counts=B.sg_get_counts(G.h),
+            A1=B.sg_get_hash_params(G.h, 1, args[1]), A2=B.sg_get_hash_params(G.h, 2, args[4]))
+        out["rep0"] = G.report(0)
+        out["rep1"] = G.report(1, 3)
+        out["rep0h"] = G.report(0 | B.SG_REPORT_HOST)
+        out["rep1h"] = G.report(1 | B.SG_REPORT_HOST, 3)
+        dens = G.density(out["rep0"][0], 2)
+        comp = G.components()
+    ref = oracle.shingling(g.row_ptr, g.col, *args)
+    assert_parity(out, ref)
+    assert dens[2] == oracle.cluster_density(g.row_ptr, g.col, out["rep0"][0], 2)[2]
+    assert np.array_equal(comp[0], oracle.connected_components(g.row_ptr, g.col)[0])
