@@ -1703,6 +1703,26 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
       a.head2 = ptr<uint32_t>(g->grp[1].head);
       a.npairs2 = g->grp[1].npairs;
       a.rows2 = P2.nrows;
+      // mode 0, s2 <= 2: the S1' nodes in length-class order for the per-node
+      // second-level constituents (built here unless pass II kept them)
+      PassOut tmp;
+      const bool nodes = mode == 0 && P2.s <= 2 && P2.nrows > 0;
+      PassOut *pc = nullptr;
+      if (nodes) {
+        if (P2.perm.p) {
+          pc = &P2;
+        } else {
+          tmp.rstart = P2.rstart;                 // borrowed (not freed through tmp)
+          tmp.rlen = P2.rlen;
+          build_row_classes(g, tmp, P2.nrows);
+          pc = &tmp;
+        }
+        a.perm2 = ptr<uint32_t>(pc->perm);
+        a.rstart2p = ptr<int64_t>(pc->rstart_p);
+        a.rlen2p = ptr<int32_t>(pc->rlen_p);
+        a.nshort2 = pc->n_split;
+        a.c2 = P2.c;
+      }
       DBuf parent, rep1, size, dlab, dnc;
       dalloc(g, parent, (size_t)a.n * 4);
       dalloc(g, rep1, (size_t)a.nk * 4);
@@ -1720,6 +1740,11 @@ sg_status report_dense_subgraphs(sg_graph *g, int32_t mode, int32_t min_size, in
       CK(cudaMemcpyAsync(&nc, dnc.p, 8, cudaMemcpyDeviceToHost, g->stream));
       sync(g);
       for (DBuf *b : {&parent, &rep1, &size, &dlab, &dnc}) dfree(g, *b);
+      if (pc == &tmp) {
+        for (DBuf *b : {&tmp.perm, &tmp.rstart_p, &tmp.rlen_p}) dfree(g, *b);
+        tmp.rstart = DBuf();
+        tmp.rlen = DBuf();
+      }
       if (n_clusters) *n_clusters = (int64_t)nc;
       return;
     }

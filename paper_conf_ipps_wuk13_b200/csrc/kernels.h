@@ -224,6 +224,13 @@ struct ReportArgs {
   const uint32_t *head2 = nullptr;      // G_II head bits
   int64_t npairs2 = 0;
   int64_t rows2 = 0;                // pass-II rows (= nk): trial t owns [t*rows2, (t+1)*rows2)
+  // mode 0, s2 <= 2: the S1' nodes in length-class order (row_classes) for
+  // the per-node second-level constituents (rows [0, nshort2) of <= 8 entries)
+  const uint32_t *perm2 = nullptr;
+  const int64_t *rstart2p = nullptr;
+  const int32_t *rlen2p = nullptr;
+  int64_t nshort2 = 0;
+  int32_t c2 = 0;
 };
 // parent/size: device uint32[n]; rep1: device uint32[nk]; labels: device
 // int32[n]; *d_nc receives the cluster count.
