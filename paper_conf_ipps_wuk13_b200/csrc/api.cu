@@ -54,7 +54,18 @@ namespace {
 // Per-handle buffer cache: freed buffers are kept and handed out again by
 // best fit, so repeated runs (bench steps, resets) allocate nothing and the
 // stream-ordered pool does not fragment and grow.
+// SG_NO_CACHE=1 (A/B hook): freed buffers go straight back to the handle's
+// stream-ordered pool (which keeps them reserved for reuse).
+bool no_cache() {
+  static const bool v = getenv("SG_NO_CACHE") != nullptr;
+  return v;
+}
+
 void cache_put(sg_graph *g, void *p, size_t bytes) {
+  if (no_cache()) {
+    cudaFreeAsync(p, g->stream);
+    return;
+  }
   g->cache.push_back({p, bytes});
   g->bytes_cached += (int64_t)bytes;
 }
