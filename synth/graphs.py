@@ -318,6 +318,12 @@ CONFIGS = {
     # AMB-20)
     "pacific640m": dict(gen=dict(n=11_000_000, n_isolated=2_403_588, m_target=640_000_000, fam_hi=3000),
                         seed=4, s1=2, c1=200, seed1=401, s2=2, c2=100, seed2=402),
+    # configs[4] sweep points at full size (the gos2m graph, other (s, c)):
+    # the extremes checked bit-exactly by oracle digests
+    "gos2m_c400": dict(gen=dict(n=2_000_000, n_isolated=437_016, m_target=56_919_738, fam_hi=3000),
+                       seed=2, s1=2, c1=400, seed1=201, s2=2, c2=400, seed2=202),
+    "gos2m_s5c50": dict(gen=dict(n=2_000_000, n_isolated=437_016, m_target=56_919_738, fam_hi=3000),
+                        seed=2, s1=5, c1=50, seed1=201, s2=5, c2=50, seed2=202),
     # small variants for parity tests (same recipe, oracle-sized)
     "small": dict(gen=dict(n=60_000, n_isolated=13_000, m_target=1_700_000, n_cliques=20,
                            cc_max=10_707, fam_hi=600),

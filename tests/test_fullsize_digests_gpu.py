@@ -1,5 +1,8 @@
 """Full-size bit-exact parity on the hub-heavy (BASELINE configs[2]) and the
-Pacific-Ocean-shaped 640M-edge (configs[3]) workloads, one GPU, against the
+Pacific-Ocean-shaped 640M-edge (configs[3]) workloads and on two extreme
+points of the trial sweep (configs[4]: s = 2, c = 400 and s = 5, c = 50 on the
+GOS-shaped graph; c = 400 runs pass II in deferred trial chunks, s = 5 uses
+the 64-bit fold ids), one GPU, against the
 digests the oracle's trial-outer run wrote (tools/oracle_digests.py ->
 tests/golden/digests_<config>.json): every pass-I column and every G_I trial,
 the S1' map, and listed pass-II columns / G_II trials, each read back trial by
@@ -28,7 +31,7 @@ def _gold(name):
 
 
 @pytest.mark.timeout(3600)
-@pytest.mark.parametrize("name", ["hub2m", "pacific640m"])
+@pytest.mark.parametrize("name", ["hub2m", "pacific640m", "gos2m_c400", "gos2m_s5c50"])
 def test_fullsize_digests(name):
     import torch
     torch.cuda.init()
