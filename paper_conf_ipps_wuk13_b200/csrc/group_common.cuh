@@ -9,6 +9,29 @@
 namespace sg {
 namespace grp {
 
+// Lanes of the warp (within vm) whose value v agrees with this lane's on the
+// low `nbits` bits: the peer mask of __match_any_sync built from nbits
+// ballots (short-latency VOTEs instead of one long-latency MATCH; ncu showed
+// the MATCH results at the head of the stall chains of the split and local
+// sorts).  Every lane of the warp must call it (converged).
+__device__ __forceinline__ uint32_t peers_by_ballot(uint32_t v, uint32_t vm, int nbits) {
+  uint32_t m = vm;
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    if (i >= nbits) break;
+    const uint32_t bit = (v >> i) & 1u;
+    const uint32_t b = __ballot_sync(0xffffffffu, bit);
+    m &= bit ? b : ~b;
+  }
+  return m;
+}
+
+__device__ __forceinline__ int bits_for(int64_t nvalues) {
+  int b = 0;
+  while (((int64_t)1 << b) < nvalues) ++b;
+  return b;
+}
+
 __device__ __forceinline__ uint32_t top_bits(uint64_t key, int bits) {
   return bits ? (uint32_t)(key >> (64 - bits)) : 0u;
 }

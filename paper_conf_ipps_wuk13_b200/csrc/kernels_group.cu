@@ -101,16 +101,15 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
   for (int b = lane; b < nb; b += 32) my[b] = 0;
   __syncwarp();
   uint32_t pr[kPerLane];
+  const int nbits = grp::bits_for(nb);
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
     const bool valid = elem_of(u) < len;
     const uint32_t vm = __ballot_sync(0xffffffffu, valid);
-    pr[u] = 0;
-    if (valid) {
-      const uint32_t b = bin_of(kk[u]);
-      pr[u] = __match_any_sync(vm, b);
-      if ((pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
-    }
+    const uint32_t b = valid ? bin_of(kk[u]) : 0u;
+    const uint32_t pm = grp::peers_by_ballot(b, vm, nbits);      // all lanes (converged)
+    pr[u] = valid ? pm : 0u;
+    if (valid && (pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
     __syncwarp();                      // the next batch's leaders read these counters
   }
   __syncthreads();
