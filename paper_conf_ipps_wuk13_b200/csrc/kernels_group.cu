@@ -90,7 +90,9 @@ struct SplitSmem {
 // [0, nb) and place them bucket-major in S.K / S.V.  obase(b) gives the output
 // position of the first pair of bin b in this chunk; S.off[b] receives
 // obase(b) - (chunk position of that pair).  Ends with a barrier.
-template <typename BIN, typename OBASE>
+// BALLOT: peer masks from ballots (measured faster for the fine split,
+// slower for the coarse scatter) or __match_any_sync.
+template <bool BALLOT, typename BIN, typename OBASE>
 __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
@@ -107,7 +109,9 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
     const bool valid = elem_of(u) < len;
     const uint32_t vm = __ballot_sync(0xffffffffu, valid);
     const uint32_t b = valid ? bin_of(kk[u]) : 0u;
-    const uint32_t pm = grp::peers_by_ballot(b, vm, nbits);      // all lanes (converged)
+    uint32_t pm = 0;
+    if (BALLOT) pm = grp::peers_by_ballot(b, vm, nbits);          // all lanes (converged)
+    else if (valid) pm = __match_any_sync(vm, b);
     pr[u] = valid ? pm : 0u;
     if (valid && (pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
     __syncwarp();                      // the next batch's leaders read these counters
@@ -325,7 +329,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
     int64_t gb = 0;
     if (threadIdx.x < nb)
       gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
-    split_place(S, len, nb, kk, vv, bin, [&](int) { return gb; });
+    split_place<false>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
     const int64_t kn = k + gridDim.x;
     if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
     emit_runs(S, len, bin, g.akeys, g.avals);
@@ -396,7 +400,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    split_place(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    split_place<true>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
     if (c0 + kChunk < n) load(c0 + kChunk);
     emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts

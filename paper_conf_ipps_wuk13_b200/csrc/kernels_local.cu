@@ -132,7 +132,7 @@ __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint1
       const bool valid = i < n;
       e[u] = valid ? (FIRST ? (uint32_t)i : (uint32_t)src[i]) : 0u;
       d[u] = valid ? (S.d20[e[u]] >> shift) & (kWDigits - 1) : (uint32_t)kWDigits;
-      m[u] = grp::peers_by_ballot(d[u], __ballot_sync(0xffffffffu, valid), kWDigitBits);
+      m[u] = __match_any_sync(0xffffffffu, d[u]);   // (ballot-built masks measured slower here)
       o[u] = 0;
       if (valid && (m[u] & lt) == 0)
         o[u] = atomicAdd(&cw[d[u] >> 1], (uint32_t)__popc(m[u]) << ((d[u] & 1) << 4));
@@ -334,9 +334,9 @@ __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *sr
   for (int pos = seg_lo + lane; pos - lane < seg_hi; pos += 32) {   // warp-uniform trip count
     const bool valid = pos < seg_hi;
     const uint32_t vm = __ballot_sync(0xffffffffu, valid);
-    const uint32_t dg = valid ? digit(S.K[src ? src[pos] : pos]) : 0u;
-    const uint32_t m = grp::peers_by_ballot(dg, vm, 8);
     if (valid) {
+      const uint32_t dg = digit(S.K[src ? src[pos] : pos]);
+      const uint32_t m = __match_any_sync(vm, dg);
       pr[pos - seg_lo] = m;
       if ((m & lt) == 0) S.cnt[dg * kLWarps + w] += (uint16_t)__popc(m);
     }
