@@ -945,8 +945,7 @@ void group_multi(sg_graph *g, int level) {
     owner_partition(g, P, ch, S, nullptr, &starts, ptr<uint64_t>(skeys), ptr<uint32_t>(svals));
     dfree(g, ch.keys);
     ch.computed = false;
-    x_alltoallv(g, skeys.p, soff.data(), rkeys.p, roff.data(), 8);
-    x_alltoallv(g, svals.p, soff.data(), rvals.p, roff.data(), 4);
+    x_alltoallv2(g, skeys.p, rkeys.p, 8, svals.p, rvals.p, 4, soff.data(), roff.data());
     st_end(g, st_x);
     dfree(g, skeys);
     dfree(g, svals);

@@ -235,41 +235,59 @@ int64_t exchange_min(sg_graph *g, int64_t v) {
   return s;
 }
 
-void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
-                 const int64_t *roff, size_t eb) {
+void x_alltoallv2(sg_graph *g, const void *send1, void *recv1, size_t eb1, const void *send2,
+                  void *recv2, size_t eb2, const int64_t *soff, const int64_t *roff) {
   Exchange *x = g->xch;
   const int R = x->world, me = x->rank;
   if (x->lb) {
     sg_loopback *lb = x->lb;
     ck(g, cudaStreamSynchronize(g->stream), "sync");     // send data complete
-    lb->dptr[(size_t)me] = send;
-    lb->doff[(size_t)me] = soff;
-    lb_barrier(g, lb);
-    for (int s = 0; s < R; ++s) {
-      const int64_t a = lb->doff[(size_t)s][me], b = lb->doff[(size_t)s][me + 1];
-      if (b > a)
-        ck(g, cudaMemcpyAsync((char *)recv + roff[s] * eb,
-                              (const char *)lb->dptr[(size_t)s] + a * eb, (size_t)(b - a) * eb,
-                              cudaMemcpyDeviceToDevice, g->stream),
-           "loopback copy");
+    for (int pass = 0; pass < 2; ++pass) {
+      const void *send = pass ? send2 : send1;
+      void *recv = pass ? recv2 : recv1;
+      const size_t eb = pass ? eb2 : eb1;
+      if (!send) continue;
+      lb->dptr[(size_t)me] = send;
+      lb->doff[(size_t)me] = soff;
+      lb_barrier(g, lb);
+      for (int s = 0; s < R; ++s) {
+        const int64_t a = lb->doff[(size_t)s][me], b = lb->doff[(size_t)s][me + 1];
+        if (b > a)
+          ck(g, cudaMemcpyAsync((char *)recv + roff[s] * eb,
+                                (const char *)lb->dptr[(size_t)s] + a * eb, (size_t)(b - a) * eb,
+                                cudaMemcpyDeviceToDevice, g->stream),
+             "loopback copy");
+      }
+      ck(g, cudaStreamSynchronize(g->stream), "sync");
+      lb_barrier(g, lb);                                        // senders may reuse buffers
     }
-    ck(g, cudaStreamSynchronize(g->stream), "sync");
-    lb_barrier(g, lb);                                        // senders may reuse buffers
     return;
   }
   if (!x->comm) fail(g, SG_ENCCL, "communicator was aborted");
+  // both arrays in one NCCL group: one collective launch per exchange
   nck(g, x->nccl->groupStart(), "ncclGroupStart");
   for (int p = 0; p < R; ++p) {
     const int64_t sc = soff[p + 1] - soff[p], rc = roff[p + 1] - roff[p];
-    if (sc > 0)
-      nck(g, x->nccl->send((const char *)send + soff[p] * eb, (size_t)sc * eb, ncclUint8, p, x->comm,
-                           g->stream), "ncclSend");
-    if (rc > 0)
-      nck(g, x->nccl->recv((char *)recv + roff[p] * eb, (size_t)rc * eb, ncclUint8, p, x->comm,
-                           g->stream), "ncclRecv");
+    for (int pass = 0; pass < 2; ++pass) {
+      const void *send = pass ? send2 : send1;
+      void *recv = pass ? recv2 : recv1;
+      const size_t eb = pass ? eb2 : eb1;
+      if (!send) continue;
+      if (sc > 0)
+        nck(g, x->nccl->send((const char *)send + soff[p] * eb, (size_t)sc * eb, ncclUint8, p, x->comm,
+                             g->stream), "ncclSend");
+      if (rc > 0)
+        nck(g, x->nccl->recv((char *)recv + roff[p] * eb, (size_t)rc * eb, ncclUint8, p, x->comm,
+                             g->stream), "ncclRecv");
+    }
   }
   nck(g, x->nccl->groupEnd(), "ncclGroupEnd");
   nccl_wait(g, "ncclSend/ncclRecv");
+}
+
+void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
+                 const int64_t *roff, size_t eb) {
+  x_alltoallv2(g, send, recv, eb, nullptr, nullptr, 0, soff, roff);
 }
 
 }  // namespace sg

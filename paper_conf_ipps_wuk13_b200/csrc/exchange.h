@@ -30,5 +30,9 @@ int64_t exchange_min(sg_graph *g, int64_t v);
 // handle's stream; returns when the transfer has completed.
 void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
                  const int64_t *roff, size_t eb);
+// Two arrays with the same element offsets (keys and generators) in one
+// exchange: one NCCL group (send2 == nullptr: one array).
+void x_alltoallv2(sg_graph *g, const void *send1, void *recv1, size_t eb1, const void *send2,
+                  void *recv2, size_t eb2, const int64_t *soff, const int64_t *roff);
 
 }  // namespace sg

@@ -17,6 +17,21 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
+def _peaks():
+    hb = 6452.8
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        hb = json.load(open(p)).get("hbm_gbs", hb)
+    hp = 3.2158e12
+    q = os.path.join(ROOT, "profiles", "int_peak.json")
+    if os.path.exists(q):
+        hp = json.load(open(q))["hash_evals_per_s"]
+    return hb, hp
+
+
+HBM_PEAK, HASH_PEAK = _peaks()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="gos2m")
@@ -60,9 +75,23 @@ def main():
                 torch.cuda.synchronize()
                 ms = e0.elapsed_time(e1) / args.steps
                 cnt = B.sg_get_counts(h)
+                # rooflines as bench.py: hash stages against the measured hash
+                # rate, grouping stages by SURVEY 8(d) bytes against copy bandwidth
+                deg = g.degrees()
+                et = {1: float(deg[deg >= s].sum()) * c, 2: float(cnt["entries2"]) * c}
+                roof = {}
+                for lv in (1, 2):
+                    th = stage.get(f"hash{lv}", 0.0) / 1e3
+                    tg = stage.get(f"group{lv}", 0.0) / 1e3
+                    if th > 0:
+                        roof[f"hash{lv}"] = round(et[lv] / th / HASH_PEAK, 4)
+                    if tg > 0:
+                        roof[f"group{lv}"] = round((32 * cnt[f"pairs{lv}"] + 8 * cnt[f"groups{lv}"]) / tg
+                                                   / 1e9 / HBM_PEAK, 4)
                 line.update(ms_per_step=round(ms, 3), edges_per_s=round(g.m / (ms / 1e3), 1),
+                            roofline_frac=roof,
                             stage_ms={k: round(stage.get(k, 0.0), 3) for k in
-                                      ("pass1", "group1", "pass2", "group2")},
+                                      ("pass1", "group1", "pass2", "group2", "hash1", "hash2")},
                             counts={k: cnt[k] for k in ("n_e", "groups1", "s1p", "entries2",
                                                         "groups2", "pairs1", "pairs2",
                                                         "chunks1", "chunks2")},
