@@ -30,13 +30,13 @@ def _gold(name):
     return json.load(open(p))
 
 
-@pytest.mark.timeout(3600)
 # the 640M-edge case takes ~10 minutes (8 of them generating the graph): run
 # with SG_FULLSIZE_640M=1 (tools/gpu_final_a.sh does; profiles/round2_pytest_gpu_final.log)
 _P640 = pytest.param("pacific640m", marks=pytest.mark.skipif(
     not os.environ.get("SG_FULLSIZE_640M"), reason="set SG_FULLSIZE_640M=1 (10 min)"))
 
 
+@pytest.mark.timeout(3600)
 @pytest.mark.parametrize("name", ["hub2m", _P640, "gos2m_c400", "gos2m_s5c50"])
 def test_fullsize_digests(name):
     import torch
