@@ -606,7 +606,6 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   a.plan.nbins = nbins;
   a.plan.nb1 = nb1;
   a.plan.npairs = npairs;
-  if (const char *e = getenv("SG_SPLIT_ATOMIC")) a.plan.split_atomic = atoi(e);
   a.plan.seg = ptr<int64_t>(S.seg);
   a.keys = keys;
   a.vals = vals;

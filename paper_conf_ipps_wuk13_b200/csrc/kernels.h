@@ -86,7 +86,6 @@ struct GroupPlan {
   int64_t chunk = 4096;            // pairs per chunk (the tables above)
   int32_t local_cap = 0;           // grouping v3: largest coarse bucket sorted by a CTA (0: default)
   int32_t fine_bits = 0;           // grouping v3: fine (counting-sort) bits after the coarse bits
-  int32_t split_atomic = 0;        // stable split: warp counters by shared atomics (A/B, SG_SPLIT_ATOMIC)
 };
 
 struct GroupArgs {

@@ -91,11 +91,8 @@ struct SplitSmem {
 // position of the first pair of bin b in this chunk; S.off[b] receives
 // obase(b) - (chunk position of that pair).  Ends with a barrier.
 // BALLOT: peer masks from ballots (measured faster for the fine split,
-// slower for the coarse scatter) or __match_any_sync.  ATOM: the warp-private
-// counters are advanced by shared-memory atomics on packed u16 pairs (the
-// counting sweep fire-and-forget, the placement with all batches' returning
-// atomics in flight) instead of read-modify-write chains with __syncwarp.
-template <bool BALLOT, bool ATOM, typename BIN, typename OBASE>
+// slower for the coarse scatter) or __match_any_sync.
+template <bool BALLOT, typename BIN, typename OBASE>
 __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
@@ -116,15 +113,8 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
     if (BALLOT) pm = grp::peers_by_ballot(b, vm, nbits);          // all lanes (converged)
     else if (valid) pm = __match_any_sync(vm, b);
     pr[u] = valid ? pm : 0u;
-    if (ATOM) {
-      if (valid && (pr[u] & lt) == 0) {
-        const int idx = w * nb + (int)b;
-        atomicAdd(reinterpret_cast<uint32_t *>(S.cnt) + (idx >> 1), (uint32_t)__popc(pr[u]) << ((idx & 1) << 4));
-      }
-    } else {
-      if (valid && (pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
-      __syncwarp();                    // the next batch's leaders read these counters
-    }
+    if (valid && (pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
+    __syncwarp();                      // the next batch's leaders read these counters
   }
   __syncthreads();
   {
@@ -150,45 +140,20 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
     if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
   __syncthreads();
-  if (ATOM) {
-    uint32_t o[kPerLane];
 #pragma unroll
-    for (int u = 0; u < kPerLane; ++u) {
-      o[u] = 0;
-      if (elem_of(u) < len && (pr[u] & lt) == 0) {
-        const int idx = w * nb + (int)bin_of(kk[u]);
-        o[u] = atomicAdd(reinterpret_cast<uint32_t *>(S.cnt) + (idx >> 1),
-                         (uint32_t)__popc(pr[u]) << ((idx & 1) << 4));
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < kPerLane; ++u) {
-      const bool valid = elem_of(u) < len;
-      const int lead = __ffs(pr[u]) - 1;
-      const uint32_t oo = __shfl_sync(0xffffffffu, o[u], lead < 0 ? 0 : lead);
-      if (valid) {
-        const int idx = w * nb + (int)bin_of(kk[u]);
-        const uint32_t p = ((oo >> ((idx & 1) << 4)) & 0xFFFFu) + __popc(pr[u] & lt);
-        S.K[p] = kk[u];
-        S.V[p] = vv[u];
-      }
-    }
-  } else {
-#pragma unroll
-    for (int u = 0; u < kPerLane; ++u) {
-      const bool valid = elem_of(u) < len;
-      const uint32_t vm = __ballot_sync(0xffffffffu, valid);
-      if (valid) {
-        const uint32_t b = bin_of(kk[u]);
-        const uint32_t rank = __popc(pr[u] & lt);
-        const uint32_t base = my[b];
-        __syncwarp(vm);
-        if (rank == 0) my[b] = (uint16_t)(base + __popc(pr[u]));
-        __syncwarp(vm);
-        const uint32_t p = base + rank;
-        S.K[p] = kk[u];
-        S.V[p] = vv[u];
-      }
+  for (int u = 0; u < kPerLane; ++u) {
+    const bool valid = elem_of(u) < len;
+    const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+    if (valid) {
+      const uint32_t b = bin_of(kk[u]);
+      const uint32_t rank = __popc(pr[u] & lt);
+      const uint32_t base = my[b];
+      __syncwarp(vm);
+      if (rank == 0) my[b] = (uint16_t)(base + __popc(pr[u]));
+      __syncwarp(vm);
+      const uint32_t p = base + rank;
+      S.K[p] = kk[u];
+      S.V[p] = vv[u];
     }
   }
   __syncthreads();
@@ -364,8 +329,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
     int64_t gb = 0;
     if (threadIdx.x < nb)
       gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
-    if (g.plan.split_atomic) split_place<false, true>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
-    else split_place<false, false>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
+    split_place<false>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
     const int64_t kn = k + gridDim.x;
     if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
     emit_runs(S, len, bin, g.akeys, g.avals);
@@ -436,8 +400,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    if (g.plan.split_atomic) split_place<true, true>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
-    else split_place<true, false>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    split_place<true>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
     if (c0 + kChunk < n) load(c0 + kChunk);
     emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts
