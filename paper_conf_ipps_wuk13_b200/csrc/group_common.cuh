@@ -26,7 +26,7 @@ __device__ __forceinline__ uint32_t peers_by_ballot(uint32_t v, uint32_t vm, int
   return m;
 }
 
-__device__ __forceinline__ int bits_for(int64_t nvalues) {
+__host__ __device__ constexpr int bits_for(int64_t nvalues) {
   int b = 0;
   while (((int64_t)1 << b) < nvalues) ++b;
   return b;

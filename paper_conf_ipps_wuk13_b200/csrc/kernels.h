@@ -102,6 +102,11 @@ struct GroupArgs {
   uint32_t *bsize;             // [c][nbins]
   uint64_t *akeys;             // [npairs] coarse-bucketed pairs
   uint32_t *avals;
+  // fused exchange (SG_DIST_PEER): owner partition writes bin d's pairs into
+  // rank d's receive buffers (device arrays of nb1 peer pointers) instead of
+  // akeys / avals
+  uint64_t *const *peer_keys = nullptr;
+  uint32_t *const *peer_vals = nullptr;
   uint64_t *bkeys;             // [npairs] final-bucketed pairs (== akeys if single-level)
   uint32_t *bvals;
   uint32_t *big_list;          // [c*nbins] bucket ids with size > 4096 (global sort)

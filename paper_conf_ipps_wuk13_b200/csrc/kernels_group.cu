@@ -91,19 +91,21 @@ struct SplitSmem {
 // position of the first pair of bin b in this chunk; S.off[b] receives
 // obase(b) - (chunk position of that pair).  Ends with a barrier.
 // BALLOT: peer masks from ballots (measured faster for the fine split,
-// slower for the coarse scatter) or __match_any_sync.
-template <bool BALLOT, typename BIN, typename OBASE>
-__device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb,
+// slower for the coarse scatter) or __match_any_sync.  NBC > 0: nb == NBC is
+// known at compile time (full 8-bit fan-out: unrolled ballots, constant loops).
+template <bool BALLOT, int NBC, typename BIN, typename OBASE>
+__device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
                                             OBASE obase) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const uint32_t lt = lanemask_lt();
+  const int nb = NBC > 0 ? NBC : nb_rt;
   uint16_t *my = S.cnt + w * nb;
   for (int b = lane; b < nb; b += 32) my[b] = 0;
   __syncwarp();
   uint32_t pr[kPerLane];
-  const int nbits = grp::bits_for(nb);
+  const int nbits = NBC > 0 ? grp::bits_for(NBC) : grp::bits_for(nb);
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
     const bool valid = elem_of(u) < len;
@@ -312,12 +314,18 @@ __device__ __forceinline__ void load_chunk(const GroupArgs &g, int64_t k, uint64
   }
 }
 
+// C8: the full 8-bit coarse fan-out (nb1 == 256), bin = the top key byte
+// (a constant shift; the generic bin costs ~10 instructions per use).
+template <bool C8>
 __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
-  const int nb = (int)g.plan.nb1;
+  const int nb = C8 ? kMaxFan : (int)g.plan.nb1;
   const int sh = pow2_shift(nb);
-  auto bin = [&](uint64_t key) { return sh >= 0 ? coarse_bin_pow2(key, sh) : coarse_bin(key, nb); };
+  auto bin = [&](uint64_t key) {
+    if (C8) return (uint32_t)(key >> 56);
+    return sh >= 0 ? coarse_bin_pow2(key, sh) : coarse_bin(key, nb);
+  };
   uint64_t kk[kPerLane];
   uint32_t vv[kPerLane];
   int64_t k = blockIdx.x;
@@ -329,16 +337,32 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
     int64_t gb = 0;
     if (threadIdx.x < nb)
       gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
-    split_place<false>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
+    split_place<false, C8 ? kMaxFan : 0>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
     const int64_t kn = k + gridDim.x;
     if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
-    emit_runs(S, len, bin, g.akeys, g.avals);
+    if (!C8 && g.peer_keys) {
+      // fused exchange: bin d = owner rank d, stored straight into its
+      // receive buffers (NVLink / NVSwitch peer stores; same device for the
+      // loopback group) at the positions the owner's grouping expects
+      for (int p = threadIdx.x; p < len; p += kSThreads) {
+        const uint64_t key = S.K[p];
+        const uint32_t d = bin(key);
+        const int64_t o = S.off[d] + p;
+        g.peer_keys[d][o] = key;
+        g.peer_vals[d][o] = S.V[p];
+      }
+    } else {
+      emit_runs(S, len, bin, g.akeys, g.avals);
+    }
     __syncthreads();
     k = kn;
   }
 }
 
 // ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
+// F8: bits == 16 with an 8-bit coarse level (the level-II plans of the 2M and
+// 640M configs): fine digit = key bits 48..55 by a constant shift.
+template <bool F8>
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -346,7 +370,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   const int64_t nb1 = g.plan.nb1;
   const int j = (int)(q1 / nb1);
   const int b1 = (int)(q1 % nb1);
-  const int bits = g.plan.bits, bits2 = g.plan.bits - g.plan.bits1;
+  const int bits = F8 ? 16 : g.plan.bits, bits2 = F8 ? 8 : g.plan.bits - g.plan.bits1;
   const int nb2 = 1 << bits2;
   const uint32_t mask2 = (uint32_t)nb2 - 1u;
   const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];
@@ -354,7 +378,10 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   const int64_t n = g.bsize1[q1];
   const uint64_t *__restrict__ K = g.akeys + sseg + st1;
   const uint32_t *__restrict__ V = g.avals + sseg + st1;
-  auto fine = [&](uint64_t key) { return top_bits(key, bits) & mask2; };
+  auto fine = [&](uint64_t key) {
+    if (F8) return (uint32_t)(key >> 48) & 0xFFu;
+    return top_bits(key, bits) & mask2;
+  };
   // fine-bucket totals (order-free), starts, sizes
   for (int i = threadIdx.x; i < nb2; i += blockDim.x) S.tot[i] = 0;
   __syncthreads();
@@ -400,7 +427,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    split_place<true>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    split_place<true, F8 ? kMaxFan : 0>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
     if (c0 + kChunk < n) load(c0 + kChunk);
     emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts
@@ -523,11 +550,14 @@ static cudaError_t split_attr(const void *fn, int *per_sm) {
 cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
+  const bool c8 = g.plan.nb1 == kMaxFan;
+  const void *fn = c8 ? (const void *)scatter_kernel<true> : (const void *)scatter_kernel<false>;
   int per_sm = 1;
-  cudaError_t e = split_attr((const void *)scatter_kernel, &per_sm);
+  cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
   const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, g.plan.nchunks);
-  scatter_kernel<<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  if (c8) scatter_kernel<true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else scatter_kernel<false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
@@ -536,10 +566,13 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   const int64_t nq1 = (int64_t)g.plan.c * g.plan.nb1;
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
   if (g.plan.bits - g.plan.bits1 > kMaxBits - kCoarseBits) return cudaErrorInvalidValue;
+  const bool f8 = g.plan.bits == 16 && g.plan.bits1 == kCoarseBits;
+  const void *fn = f8 ? (const void *)scatter2_kernel<true> : (const void *)scatter2_kernel<false>;
   int per_sm = 1;
-  cudaError_t e = split_attr((const void *)scatter2_kernel, &per_sm);
+  cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
-  scatter2_kernel<<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  if (f8) scatter2_kernel<true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else scatter2_kernel<false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }

@@ -195,12 +195,15 @@ __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n
   return __any_sync(0xffffffffu, bad);
 }
 
+// BITS > 0: the plan's bucket bits known at compile time (16: the level-II
+// plans of the 2M / 640M configs), so the sort digits are constant shifts.
+template <int BITS>
 __global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   WarpSmem &S = reinterpret_cast<WarpSmem *>(smraw)[wl];
   const int64_t nq = (int64_t)g.plan.c * g.plan.nbins;
-  const int bits = g.plan.bits;
+  const int bits = BITS > 0 ? BITS : g.plan.bits;
   const int64_t obase = g.plan.seg[0];     // scratch -> output position
   const int64_t nwarps = (int64_t)gridDim.x * kWWarps;
   for (int64_t q = (int64_t)blockIdx.x * kWWarps + wl; q < nq; q += nwarps) {
@@ -229,15 +232,17 @@ __global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __gri
     __syncwarp();
     // one sweep: the 20 sort bits of each key and both digit histograms
     // (packed 16-bit counters, order-free); the values are prefetched into L1
-    for (int i0 = 0; i0 < n; i0 += 128) {
-      uint64_t k4[4];
+    // eight key loads in flight per lane (ncu: the sweep's first use of a
+    // key headed the kernel's stall list with four)
+    for (int i0 = 0; i0 < n; i0 += 256) {
+      uint64_t k4[8];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < 8; ++u) {
         const int i = i0 + u * 32 + lane;
         k4[u] = i < n ? Kg[i] : 0ull;
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < 8; ++u) {
         const int i = i0 + u * 32 + lane;
         if (i < n) {
           const uint32_t d20 = (uint32_t)((k4[u] << bits) >> 44);
@@ -530,16 +535,18 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   // warp tier over all buckets
   {
     const size_t smem = sizeof(WarpSmem) * kWWarps;
-    cudaError_t e = cudaFuncSetAttribute(warp_local_kernel,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const bool b16 = g.plan.bits == 16;
+    const void *fn = b16 ? (const void *)warp_local_kernel<16> : (const void *)warp_local_kernel<0>;
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, warp_local_kernel, kWWarps * 32, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kWWarps * 32, smem);
     if (e != cudaSuccess) return e;
     per_sm = std::max(per_sm, 1);
     const int64_t want = (nq + kWWarps - 1) / kWWarps;
     const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, want);
-    warp_local_kernel<<<grid, kWWarps * 32, smem, st>>>(g);
+    if (b16) warp_local_kernel<16><<<grid, kWWarps * 32, smem, st>>>(g);
+    else warp_local_kernel<0><<<grid, kWWarps * 32, smem, st>>>(g);
     ++g_launches;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
