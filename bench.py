@@ -227,7 +227,7 @@ def bench_ours(args, rank, world, local_rank):
     stream = torch.cuda.Stream()           # a non-default stream shared with the library
     torch.cuda.set_stream(stream)
     dinfo = {"rank": rank, "world": world, "device": local_rank, "stream": stream.cuda_stream,
-             "exchange": args.exchange}
+             "exchange": args.exchange, "peer": args.peer}
     shard_mode = args.shard == "components" and world > 1
     if shard_mode:
         # pClust's decomposition (N3): whole connected components per rank,
@@ -389,7 +389,9 @@ def bench_ours(args, rank, world, local_rank):
                          % ((g.row_ptr.nbytes + g.col.nbytes) / 1e6),
                    "parallelism": (f"connected-component shards x{world} (no exchange)" if shard_mode
                                    else f"vertex-range shards x{world}"),
-                   "exchange": bool(counts["exchange"]), "comm_world": counts["world"]},
+                   "exchange": bool(counts["exchange"]), "comm_world": counts["world"],
+                   "exchange_transport": ("peer stores (SG_DIST_PEER)" if args.peer else "nccl send/recv")
+                   if counts["exchange"] else None},
         "stage_ms": {k: round(v, 3) for k, v in stage_ms.items() if v > 0},
         "roofline": dom, "roofline_stages": rt, "peak_source": pk["src"], "phase3": phase3,
         "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches * args.steps,
@@ -489,6 +491,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-nnz", type=int, default=1_500_000)
     ap.add_argument("--ref-sample-nnz", type=int, default=1_500_000)
+    ap.add_argument("--peer", action="store_true",
+                    help="fused exchange: the owner split stores pairs straight into the owners' receive "
+                         "buffers over NVLink peer memory (SG_DIST_PEER) instead of NCCL send/recv")
     ap.add_argument("--exchange", action="store_true",
                     help="N=1: route the pairs through the NCCL exchange path anyway (a 1-rank communicator)")
     ap.add_argument("--dry-run", action="store_true", help="CPU check of the multi-rank launch logic")

@@ -69,9 +69,23 @@ typedef struct sg_dist {
     uint32_t flags;            /* SG_DIST_EXCHANGE: run the owner-routed exchange path even */
                                /* at world == 1 (a one-rank NCCL communicator or loopback   */
                                /* group; exercises the multi-GPU transport on one GPU)      */
+                               /* SG_DIST_PEER: fused exchange (below)                      */
 } sg_dist;
 
 #define SG_DIST_EXCHANGE 0x1u
+/* SG_DIST_PEER — fused partition + transfer over peer memory (SURVEY §8(f)
+ * N2): every rank exposes one receive buffer per level to all
+ * ranks (NCCL backend: CUDA IPC handles exchanged over the communicator, the
+ * peers' buffers mapped into this process — NVLink / NVSwitch P2P; loopback:
+ * the device pointers of the other virtual ranks), and the owner-partition
+ * kernel stores each <shingle, generator> pair straight into its owner's
+ * receive buffer at its final position, so no send buffer is written and no
+ * NCCL send / recv runs.  The received layout, and hence every output, is
+ * identical to the send / recv path.  Ranks synchronise with a barrier
+ * before a chunk is written (the owners finished grouping the previous one)
+ * and after (all pairs delivered).  Needs P2P access between the ranks'
+ * devices (NCCL backend) — SG_ECUDA otherwise. */
+#define SG_DIST_PEER 0x2u
 
 /* ------------------------------------------------------------------------ */
 /* shingle_graph_create — ingest an unweighted G(V, E) given as adjacency   */

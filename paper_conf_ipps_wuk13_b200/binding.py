@@ -42,6 +42,7 @@ class sg_dist(C.Structure):
 
 
 SG_DIST_EXCHANGE = 0x1
+SG_DIST_PEER = 0x2
 
 
 _lib = None
@@ -131,7 +132,8 @@ def shingle_graph_create(row_ptr, col, validate: bool = True, dist: Optional[dic
     if dist is not None:
         d = sg_dist(int(dist.get("rank", 0)), int(dist.get("world", 1)), int(dist.get("device", 0)),
                     dist.get("stream"), None, dist.get("loopback"),
-                    SG_DIST_EXCHANGE if dist.get("exchange") else 0)
+                    (SG_DIST_EXCHANGE if dist.get("exchange") else 0) |
+                    (SG_DIST_PEER if dist.get("peer") else 0))
         uid = dist.get("nccl_uid")
         if uid is not None:
             d._uid_buf = C.create_string_buffer(bytes(uid), 128)

@@ -222,6 +222,7 @@ void free_pass(sg_graph *g, PassOut &p) {
   for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid, &p.perm, &p.rstart_p, &p.rlen_p}) dfree(g, *b);
   for (auto &ch : p.chunks) {
     dfree(g, ch.keys);
+    dfree(g, ch.kbin);
     dfree(g, ch.ctr);
     if (ch.done) cudaEventDestroy(ch.done);
   }
@@ -419,6 +420,10 @@ void build_row_classes(sg_graph *g, PassOut &P, int64_t nrows) {
 void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_side = false) {
   if (!on_side) st_begin(g, st_hash);   // side chunks: timed on the side stream below
   dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
+  // top key bytes for the coarse histogram (1 B instead of 8 B per pair):
+  // single rank, stable grouping, rows in generator order
+  const bool want_kbin = !g->xch && use_group_v1() && P.perm.p == nullptr && !getenv("SG_NO_KBIN");
+  if (want_kbin) dalloc(g, ch.kbin, (size_t)ch.nt * (size_t)P.key_stride);
   DBuf &ctr = ch.ctr;
   dalloc(g, ctr, 16);
   CK(cudaMemsetAsync(ctr.p, 0, 16, g->stream));
@@ -443,6 +448,7 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_s
   a.s = P.s;
   a.seed = P.seed;
   a.keys = ptr<uint64_t>(ch.keys);
+  a.kbin = want_kbin ? ptr<uint8_t>(ch.kbin) : nullptr;
   a.key_stride = P.key_stride;
   a.counter = ptr<unsigned long long>(ctr);
   a.hub_counter = a.counter + 1;
@@ -564,7 +570,7 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
                   int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,
                   const uint32_t *rowid, uint32_t val_base, Groups &out, uint64_t *okeys,
                   GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter,
-                  int st_local) {
+                  int st_local, const uint8_t *kbin = nullptr) {
   int64_t maxseg = 0, npairs = 0;
   for (int j = 0; j < nt; ++j) {
     const int64_t L = seg_all[(size_t)t0 + j + 1] - seg_all[(size_t)t0 + j];
@@ -608,6 +614,7 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   a.plan.npairs = npairs;
   a.plan.seg = ptr<int64_t>(S.seg);
   a.keys = keys;
+  a.kbin = kbin;
   a.vals = vals;
   a.rowid = rowid;
   a.val_base = val_base;
@@ -733,10 +740,11 @@ void group_pieces_b(sg_graph *g, const uint64_t *keys, const std::vector<Piece> 
 void group_any(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &pieces, int32_t t0,
                int32_t nt, const std::vector<int64_t> &seg_all, const uint32_t *vals,
                const uint32_t *rowid, uint32_t val_base, Groups &out, uint64_t *okeys,
-               GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter, int st_local) {
+               GroupScratch &S, DBuf *free_after_scatter, int st_hist, int st_scatter, int st_local,
+               const uint8_t *kbin = nullptr) {
   if (use_group_v1())
     group_pieces(g, keys, pieces, t0, nt, seg_all, vals, rowid, val_base, out, okeys, S,
-                 free_after_scatter, st_hist, st_scatter, st_local);
+                 free_after_scatter, st_hist, st_scatter, st_local, kbin);
   else
     group_pieces_b(g, keys, pieces, t0, nt, seg_all, vals, rowid, val_base, out, okeys, S,
                    free_after_scatter, st_hist, st_scatter, st_local);
@@ -828,9 +836,13 @@ void assign_s1p_index(sg_graph *g, PassOut &P) {
 // canonical key order is rank-major).  Virtual trial vt = tl * nblk + b.
 // Phase `starts == nullptr`: counts only (mine[vt * R + d]).  Otherwise the
 // pairs are written dest-major (then vt, then row order) into skeys / svals.
+// Fused exchange (SG_DIST_PEER): peer_k / peer_v are device arrays of the
+// owners' receive buffers and `starts` are positions in them; the pairs are
+// stored there directly (skeys / svals unused).
 void owner_partition(sg_graph *g, PassOut &P, KeyChunk &ch, GroupScratch &S,
                      std::vector<int64_t> *mine, const std::vector<int64_t> *starts,
-                     uint64_t *skeys, uint32_t *svals) {
+                     uint64_t *skeys, uint32_t *svals, uint64_t *const *peer_k = nullptr,
+                     uint32_t *const *peer_v = nullptr) {
   const int R = g->world;
   const std::vector<int64_t> &Bk = P.blocks;
   const int nblk = (int)Bk.size() - 1;
@@ -872,8 +884,23 @@ void owner_partition(sg_graph *g, PassOut &P, KeyChunk &ch, GroupScratch &S,
   a.plan.seg = ptr<int64_t>(S.seg);
   a.akeys = skeys;
   a.avals = svals;
+  a.peer_keys = peer_k;
+  a.peer_vals = peer_v;
   CK(group_scatter(a, g->num_sms, g->stream));
 }
+
+// Receive buffers of the fused exchange: cudaMalloc'd (IPC-exportable), one
+// pair per level, mapped by every rank; released on every exit path.
+struct PeerRecv {
+  void *k = nullptr, *v = nullptr;
+  std::vector<void *> opened;
+  DBuf dk, dv;                 // device arrays of the R peer pointers
+  ~PeerRecv() {
+    for (void *p : opened) cudaIpcCloseMemHandle(p);
+    if (k) cudaFree(k);
+    if (v) cudaFree(v);
+  }
+};
 
 // Exchange + grouping of one level on a multi-rank handle.
 void group_multi(sg_graph *g, int level) {
@@ -915,6 +942,31 @@ void group_multi(sg_graph *g, int level) {
   dalloc(g, out.okeys, (size_t)out.npairs * 8);
   dalloc(g, out.head, (size_t)((out.npairs + 31) / 32) * 4);
   CK(cudaMemsetAsync(out.head.p, 0, out.head.bytes, g->stream));
+  // fused exchange: one receive buffer per rank, sized for its largest chunk
+  PeerRecv pr;
+  if (g->peer_xch) {
+    int64_t rcap = 1;
+    for (size_t k = 0; k < P.chunks.size(); ++k) {
+      const int64_t n = (int64_t)P.chunks[k].nt * nblk * R;
+      int64_t t = 0;
+      for (int s = 0; s < R; ++s)
+        for (int64_t vt = 0; vt < (int64_t)P.chunks[k].nt * nblk; ++vt)
+          t += all[k][(size_t)(s * n + vt * R + me)];
+      rcap = std::max(rcap, t);
+    }
+    CK(cudaMalloc(&pr.k, (size_t)rcap * 8));
+    CK(cudaMalloc(&pr.v, (size_t)rcap * 4));
+    void *mine2[2] = {pr.k, pr.v};
+    std::vector<void *> peers;
+    x_share_buffers(g, mine2, 2, peers, pr.opened);
+    std::vector<void *> pk((size_t)R), pv((size_t)R);
+    for (int r = 0; r < R; ++r) {
+      pk[(size_t)r] = peers[(size_t)r * 2];
+      pv[(size_t)r] = peers[(size_t)r * 2 + 1];
+    }
+    upload(g, pr.dk, pk.data(), (size_t)R * sizeof(void *));
+    upload(g, pr.dv, pv.data(), (size_t)R * sizeof(void *));
+  }
   // phase 2: per chunk, partition to send buffers, all-to-all, group
   for (size_t k = 0; k < P.chunks.size(); ++k) {
     KeyChunk &ch = P.chunks[k];
@@ -937,18 +989,49 @@ void group_multi(sg_graph *g, int level) {
       roff[(size_t)s + 1] = roff[(size_t)s] + t;
     }
     DBuf skeys, svals, rkeys, rvals;
-    dalloc(g, skeys, (size_t)soff[(size_t)R] * 8);
-    dalloc(g, svals, (size_t)soff[(size_t)R] * 4);
-    dalloc(g, rkeys, (size_t)roff[(size_t)R] * 8);
-    dalloc(g, rvals, (size_t)roff[(size_t)R] * 4);
-    st_begin(g, st_x);
-    owner_partition(g, P, ch, S, nullptr, &starts, ptr<uint64_t>(skeys), ptr<uint32_t>(svals));
-    dfree(g, ch.keys);
-    ch.computed = false;
-    x_alltoallv2(g, skeys.p, rkeys.p, 8, svals.p, rvals.p, 4, soff.data(), roff.data());
-    st_end(g, st_x);
-    dfree(g, skeys);
-    dfree(g, svals);
+    uint64_t *rk = nullptr;
+    uint32_t *rv = nullptr;
+    if (g->peer_xch) {
+      // positions in the owners' receive buffers (their layout: source-major,
+      // then virtual trial, then row order — the send / recv layout)
+      std::vector<int64_t> pst((size_t)nvt * R);
+      for (int d = 0; d < R; ++d) {
+        int64_t run = 0;
+        for (int s = 0; s < me; ++s)
+          for (int vt = 0; vt < nvt; ++vt) run += all[k][(size_t)(s * n + (int64_t)vt * R + d)];
+        for (int vt = 0; vt < nvt; ++vt) {
+          pst[(size_t)vt * R + d] = run;
+          run += all[k][(size_t)(me * n + (int64_t)vt * R + d)];
+        }
+      }
+      st_begin(g, st_x);
+      x_barrier(g);                    // every owner has grouped its previous chunk
+      owner_partition(g, P, ch, S, nullptr, &pst, nullptr, nullptr,
+                      reinterpret_cast<uint64_t *const *>(pr.dk.p),
+                      reinterpret_cast<uint32_t *const *>(pr.dv.p));
+      dfree(g, ch.keys);
+      ch.computed = false;
+      sync(g);
+      x_barrier(g);                    // every pair of this chunk is delivered
+      st_end(g, st_x);
+      rk = static_cast<uint64_t *>(pr.k);
+      rv = static_cast<uint32_t *>(pr.v);
+    } else {
+      dalloc(g, skeys, (size_t)soff[(size_t)R] * 8);
+      dalloc(g, svals, (size_t)soff[(size_t)R] * 4);
+      dalloc(g, rkeys, (size_t)roff[(size_t)R] * 8);
+      dalloc(g, rvals, (size_t)roff[(size_t)R] * 4);
+      st_begin(g, st_x);
+      owner_partition(g, P, ch, S, nullptr, &starts, ptr<uint64_t>(skeys), ptr<uint32_t>(svals));
+      dfree(g, ch.keys);
+      ch.computed = false;
+      x_alltoallv2(g, skeys.p, rkeys.p, 8, svals.p, rvals.p, 4, soff.data(), roff.data());
+      st_end(g, st_x);
+      dfree(g, skeys);
+      dfree(g, svals);
+      rk = ptr<uint64_t>(rkeys);
+      rv = ptr<uint32_t>(rvals);
+    }
     // received pieces in canonical generator order: trial, row block, source
     std::vector<Piece> pieces;
     for (int tl = 0; tl < ch.nt; ++tl)
@@ -960,12 +1043,18 @@ void group_multi(sg_graph *g, int level) {
           const int64_t len = all[k][(size_t)(s * n + (int64_t)vt * R + me)];
           if (len > 0) pieces.push_back(Piece{tl, o, len, 0});
         }
-    group_any(g, ptr<uint64_t>(rkeys), pieces, ch.t0, ch.nt, out.seg, ptr<uint32_t>(rvals),
+    group_any(g, rk, pieces, ch.t0, ch.nt, out.seg, rv,
                  nullptr, 0, out, ptr<uint64_t>(out.okeys), S, nullptr,
                  level == 0 ? kStHist1 : kStHist2, level == 0 ? kStScatter1 : kStScatter2,
                  level == 0 ? kStLocal1 : kStLocal2);
-    dfree(g, rkeys);
-    dfree(g, rvals);
+    if (rkeys.p) dfree(g, rkeys);
+    if (rvals.p) dfree(g, rvals);
+  }
+  if (g->peer_xch) {
+    sync(g);                           // this rank's reads of its receive buffer are done
+    x_release_buffers(g, pr.opened);   // barrier: no peer writes any more
+    dfree(g, pr.dk);
+    dfree(g, pr.dv);
   }
   free_scratch(g, S);
   g->pairs_global[level] = exchange_sum(g, out.npairs);
@@ -1239,7 +1328,10 @@ sg_status shingle_graph_create(int64_t n, int64_t nnz, const int64_t *row_ptr, c
     uint64_t thr = UINT64_MAX;
     CK(cudaMemPoolSetAttribute(g->pool, cudaMemPoolAttrReleaseThreshold, &thr));
     ingest(g, n, nnz, row_ptr, rp_host, col, devptr, validate, (flags & SG_HOST_CSR) != 0);
-    if (g->world > 1 || (dist && (dist->flags & SG_DIST_EXCHANGE))) g->xch = exchange_create(g, dist);
+    if (g->world > 1 || (dist && (dist->flags & SG_DIST_EXCHANGE))) {
+      g->xch = exchange_create(g, dist);
+      g->peer_xch = (dist->flags & SG_DIST_PEER) != 0;
+    }
     sync(g);
     g->launch_base = g_launches.load();
     g->state = kCreated;
@@ -1433,7 +1525,9 @@ sg_status group_by_shingle(sg_graph *g) {
           pieces.push_back(Piece{tl, (int64_t)tl * P.key_stride, P.nrows, 0});
         group_any(g, ptr<uint64_t>(ch.keys), pieces, ch.t0, ch.nt, out.seg, nullptr, rowid, base,
                      out, nullptr, S, &ch.keys, level == 0 ? kStHist1 : kStHist2,
-                     level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2);
+                     level == 0 ? kStScatter1 : kStScatter2, level == 0 ? kStLocal1 : kStLocal2,
+                     ch.kbin.p ? ptr<uint8_t>(ch.kbin) : nullptr);
+        dfree(g, ch.kbin);
         ch.computed = false;
       }
       free_scratch(g, S);
@@ -1475,6 +1569,7 @@ void shingle_graph_destroy(sg_graph *g) {
     for (DBuf *b : {&p.A, &p.B, &p.rstart, &p.rlen, &p.rowid}) rel(b->p);
     for (auto &ch : p.chunks) {
       rel(ch.keys.p);
+      rel(ch.kbin.p);
       rel(ch.ctr.p);
     }
     for (DBuf *b : {&g->grp[l].members, &g->grp[l].head, &g->grp[l].okeys}) rel(b->p);

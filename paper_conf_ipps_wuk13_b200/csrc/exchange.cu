@@ -290,6 +290,62 @@ void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
   x_alltoallv2(g, send, recv, eb, nullptr, nullptr, 0, soff, roff);
 }
 
+void x_barrier(sg_graph *g) {
+  Exchange *x = g->xch;
+  if (x->lb) {
+    lb_barrier(g, x->lb);
+    return;
+  }
+  int64_t one = 1;
+  std::vector<int64_t> all((size_t)x->world);
+  x_allgather_i64(g, &one, 1, all.data());     // returns after every rank contributed
+}
+
+void x_share_buffers(sg_graph *g, void *const *mine, int nbuf, std::vector<void *> &all,
+                     std::vector<void *> &opened) {
+  Exchange *x = g->xch;
+  const int R = x->world, me = x->rank;
+  all.assign((size_t)R * nbuf, nullptr);
+  opened.clear();
+  if (x->lb) {
+    std::vector<int64_t> v((size_t)nbuf), a((size_t)R * nbuf);
+    for (int i = 0; i < nbuf; ++i) v[(size_t)i] = (int64_t)(intptr_t)mine[i];
+    x_allgather_i64(g, v.data(), nbuf, a.data());
+    for (size_t i = 0; i < a.size(); ++i) all[i] = (void *)(intptr_t)a[i];
+    return;
+  }
+  // NCCL backend: one process per GPU; IPC handles travel as int64 words
+  static_assert(sizeof(cudaIpcMemHandle_t) % 8 == 0, "IPC handle size");
+  const int W = (int)(sizeof(cudaIpcMemHandle_t) / 8);
+  std::vector<int64_t> v((size_t)nbuf * W), a((size_t)R * nbuf * W);
+  for (int i = 0; i < nbuf; ++i) {
+    cudaIpcMemHandle_t h;
+    memset(&h, 0, sizeof h);
+    if (mine[i]) ck(g, cudaIpcGetMemHandle(&h, mine[i]), "cudaIpcGetMemHandle");
+    memcpy(v.data() + (size_t)i * W, &h, sizeof h);
+  }
+  x_allgather_i64(g, v.data(), (int64_t)nbuf * W, a.data());
+  for (int r = 0; r < R; ++r)
+    for (int i = 0; i < nbuf; ++i) {
+      if (r == me) {
+        all[(size_t)r * nbuf + i] = mine[i];
+        continue;
+      }
+      cudaIpcMemHandle_t h;
+      memcpy(&h, a.data() + ((size_t)r * nbuf + i) * W, sizeof h);
+      void *p = nullptr;
+      ck(g, cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+      all[(size_t)r * nbuf + i] = p;
+      opened.push_back(p);
+    }
+}
+
+void x_release_buffers(sg_graph *g, std::vector<void *> &opened) {
+  x_barrier(g);
+  for (void *p : opened) cudaIpcCloseMemHandle(p);
+  opened.clear();
+}
+
 }  // namespace sg
 
 // ---------------------------------------------------------------- C ABI

@@ -10,6 +10,8 @@
 //    memcpys.  It exercises the whole multi-rank path on a single GPU.
 #pragma once
 
+#include <vector>
+
 #include "sg_internal.cuh"
 
 namespace sg {
@@ -30,6 +32,19 @@ int64_t exchange_min(sg_graph *g, int64_t v);
 // handle's stream; returns when the transfer has completed.
 void x_alltoallv(sg_graph *g, const void *send, const int64_t *soff, void *recv,
                  const int64_t *roff, size_t eb);
+
+// ---- fused exchange over peer memory (SG_DIST_PEER)
+// Barrier over the ranks (host: returns when every rank has called it).
+void x_barrier(sg_graph *g);
+// Publish `nbuf` device buffers of this rank (allocated with cudaMalloc) and
+// map every rank's: all[r * nbuf + i] is rank r's buffer i, usable by this
+// rank's kernels (NCCL backend: CUDA IPC handles exchanged over the
+// communicator and opened here; loopback: the peers' pointers, same device).
+// `opened` receives the mappings this rank must release.
+void x_share_buffers(sg_graph *g, void *const *mine, int nbuf, std::vector<void *> &all,
+                     std::vector<void *> &opened);
+// Barrier (no rank still writes into a peer buffer), then unmap `opened`.
+void x_release_buffers(sg_graph *g, std::vector<void *> &opened);
 // Two arrays with the same element offsets (keys and generators) in one
 // exchange: one NCCL group (send2 == nullptr: one array).
 void x_alltoallv2(sg_graph *g, const void *send1, void *recv1, size_t eb1, const void *send2,

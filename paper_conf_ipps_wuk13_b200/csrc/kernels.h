@@ -45,6 +45,8 @@ struct MinhashArgs {
   unsigned long long *counter;    // zeroed device counter (row tiles)
   unsigned long long *hub_counter;  // zeroed device counter (hub-row blocks)
   int32_t tile_rows = 8;          // rows per warp tile: 8 (long rows) or 16 (short rows)
+  uint8_t *kbin = nullptr;        // [nt][key_stride] top key byte (the grouping's coarse bin,
+                                  // read by hist_kernel instead of the 8-B keys) or nullptr
 };
 constexpr int kRowTile = 16;      // key_stride granule (multiple of every tile size)
 inline int64_t key_stride_for(int64_t nrows) { return (nrows + kRowTile - 1) / kRowTile * kRowTile; }
@@ -91,6 +93,7 @@ struct GroupPlan {
 struct GroupArgs {
   GroupPlan plan;
   const uint64_t *keys;        // [npairs] pre-group keys (per-trial segments)
+  const uint8_t *kbin = nullptr;   // top byte of each key, same indexing (or nullptr)
   const uint32_t *vals;        // explicit generator values, or nullptr:
   const uint32_t *rowid;       //   val = rowid[i - seg[j]] if rowid, else
   uint32_t val_base;           //   val = val_base + (i - seg[j])
@@ -132,6 +135,7 @@ cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, c
                          int32_t c, cudaStream_t st);
 
 int64_t group_local_capacity();
+int split_atomic();              // SG_SPLIT_ATOMIC: atomic split ranking (1: fine split, 2: + coarse)
 int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
 // Bucket plan for trial segments of at most `maxseg` pairs.
@@ -178,6 +182,7 @@ cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, c
                          int32_t c, cudaStream_t st);
 
 int64_t group_local_capacity();
+int split_atomic();              // SG_SPLIT_ATOMIC: atomic split ranking (1: fine split, 2: + coarse)
 int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
 // Bucket plan for trial segments of at most `maxseg` pairs.

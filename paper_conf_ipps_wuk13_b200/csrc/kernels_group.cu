@@ -12,9 +12,12 @@
 //                 contiguous per-bucket runs (coalesced stores);
 //   4. scatter2 : two-level plans only: one CTA per coarse bucket splits it
 //                 stably by the next <= 8 bits with the same engine.
-// Stability matters: the input of every trial is in generator order, so the
+// Stability pays: the input of every trial is in generator order, so the
 // members of one group (equal keys) arrive in ascending order and the local
-// sort never has to sort a group by member.
+// sort rarely has to sort a group by member.  Correctness does not depend on
+// it: the local sorts verify the full (key, member) order of every bucket and
+// repair the runs that violate it (the fine split ranks by shared atomics,
+// whose lane order the hardware does not promise).
 #include <algorithm>
 #include <cstdlib>
 
@@ -93,7 +96,13 @@ struct SplitSmem {
 // BALLOT: peer masks from ballots (measured faster for the fine split,
 // slower for the coarse scatter) or __match_any_sync.  NBC > 0: nb == NBC is
 // known at compile time (full 8-bit fan-out: unrolled ballots, constant loops).
-template <bool BALLOT, int NBC, typename BIN, typename OBASE>
+// AT: no peer masks at all — every pair counts and takes its slot with its
+// own shared atomic on the warp's packed u16 counters.  Pairs of one warp
+// are visited batch by batch in input order; within one warp instruction the
+// order of conflicting lanes is the hardware's (tools/atom_order.cu measures
+// it).  The final sorts verify the full (key, member) order and repair any
+// run that is out of it, so the result never depends on that order.
+template <bool BALLOT, int NBC, bool AT, typename BIN, typename OBASE>
 __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
@@ -102,10 +111,19 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
   const uint32_t lt = lanemask_lt();
   const int nb = NBC > 0 ? NBC : nb_rt;
   uint16_t *my = S.cnt + w * nb;
+  uint32_t *cw = reinterpret_cast<uint32_t *>(S.cnt);
   for (int b = lane; b < nb; b += 32) my[b] = 0;
   __syncwarp();
   uint32_t pr[kPerLane];
   const int nbits = NBC > 0 ? grp::bits_for(NBC) : grp::bits_for(nb);
+  if (AT) {
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u)
+      if (elem_of(u) < len) {
+        const int idx = w * nb + (int)bin_of(kk[u]);
+        atomicAdd(cw + (idx >> 1), 1u << ((idx & 1) << 4));
+      }
+  } else {
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
     const bool valid = elem_of(u) < len;
@@ -117,6 +135,7 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
     pr[u] = valid ? pm : 0u;
     if (valid && (pr[u] & lt) == 0) my[b] += (uint16_t)__popc(pr[u]);   // lowest peer leads
     __syncwarp();                      // the next batch's leaders read these counters
+  }
   }
   __syncthreads();
   {
@@ -142,6 +161,26 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
     if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
   __syncthreads();
+  if (AT) {
+    uint32_t o[kPerLane];
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u) {
+      o[u] = 0;
+      if (elem_of(u) < len) {
+        const int idx = w * nb + (int)bin_of(kk[u]);
+        o[u] = atomicAdd(cw + (idx >> 1), 1u << ((idx & 1) << 4)) >> ((idx & 1) << 4);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u)
+      if (elem_of(u) < len) {
+        const uint32_t p = o[u] & 0xFFFFu;
+        S.K[p] = kk[u];
+        S.V[p] = vv[u];
+      }
+    __syncthreads();
+    return;
+  }
 #pragma unroll
   for (int u = 0; u < kPerLane; ++u) {
     const bool valid = elem_of(u) < len;
@@ -217,6 +256,44 @@ __global__ void __launch_bounds__(kHThreads) hist_kernel(const __grid_constant__
     }
 #pragma unroll
     for (int u = 0; u < kHPer; ++u) kk[u] = nx[u];
+  }
+}
+
+// The same histogram from the min-hash kernels' top-key-byte array (1 B per
+// pair instead of the 8-B key; power-of-two coarse fan-outs of <= 256 bins):
+// one 4-byte load per thread and chunk.
+__global__ void __launch_bounds__(kHThreads) hist_bytes_kernel(const __grid_constant__ GroupArgs g) {
+  __shared__ uint32_t hist[kMaxFan];
+  const int nb = (int)g.plan.nb1;
+  const int sh = 8 - grp::bits_for(nb);
+  const int64_t k0 = (int64_t)blockIdx.x * kHistChunks;
+  const int64_t k1 = min(k0 + kHistChunks, g.plan.nchunks);
+  for (int i = threadIdx.x; i < kMaxFan; i += kHThreads) hist[i] = 0;
+  auto load = [&](int64_t k) -> uint32_t {
+    const int len = g.plan.chunk_len[k];
+    const uint8_t *__restrict__ kb = g.kbin + g.plan.chunk_in0[k];
+    const int i = 4 * threadIdx.x;
+    if (i + 4 <= len) return *reinterpret_cast<const uint32_t *>(kb + i);
+    uint32_t w = 0;
+    for (int x = 0; x < 4 && i + x < len; ++x) w |= (uint32_t)kb[i + x] << (8 * x);
+    return w;
+  };
+  uint32_t cur = k0 < k1 ? load(k0) : 0u;
+  __syncthreads();
+  for (int64_t k = k0; k < k1; ++k) {
+    const uint32_t nxt = k + 1 < k1 ? load(k + 1) : 0u;   // in flight while counting
+    const int len = g.plan.chunk_len[k];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (4 * (int)threadIdx.x + x < len) atomicAdd(&hist[((cur >> (8 * x)) & 0xFFu) >> sh], 1u);
+    __syncthreads();
+    uint32_t *out = g.counts + k * nb;
+    for (int i = threadIdx.x; i < nb; i += kHThreads) {
+      out[i] = hist[i];
+      hist[i] = 0;
+    }
+    __syncthreads();
+    cur = nxt;
   }
 }
 
@@ -316,7 +393,7 @@ __device__ __forceinline__ void load_chunk(const GroupArgs &g, int64_t k, uint64
 
 // C8: the full 8-bit coarse fan-out (nb1 == 256), bin = the top key byte
 // (a constant shift; the generic bin costs ~10 instructions per use).
-template <bool C8>
+template <bool C8, bool AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -337,7 +414,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
     int64_t gb = 0;
     if (threadIdx.x < nb)
       gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
-    split_place<false, C8 ? kMaxFan : 0>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
+    split_place<false, C8 ? kMaxFan : 0, AT>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
     const int64_t kn = k + gridDim.x;
     if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
     if (!C8 && g.peer_keys) {
@@ -362,7 +439,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
 // ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
 // F8: bits == 16 with an 8-bit coarse level (the level-II plans of the 2M and
 // 640M configs): fine digit = key bits 48..55 by a constant shift.
-template <bool F8>
+template <bool F8, bool AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -427,7 +504,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    split_place<true, F8 ? kMaxFan : 0>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    split_place<true, F8 ? kMaxFan : 0, AT>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
     if (c0 + kChunk < n) load(c0 + kChunk);
     emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts
@@ -480,6 +557,23 @@ __global__ void sum_i32_kernel(const int32_t *__restrict__ a, int64_t n, unsigne
 
 }  // namespace
 
+// Ranking by per-pair shared atomics (split_place<..., AT = true>) in the
+// fine split (default; SG_SPLIT_ATOMIC=0: ballot-built peer masks) and, with
+// SG_SPLIT_ATOMIC=2, in the coarse scatter as well.  The local sorts verify
+// and repair the (key, member) order, so the outputs are the same either
+// way; on the B200 conflicting lanes are served in lane order
+// (tools/atom_order.cu: 0 of 1.55e8 warp-instructions out of order), so the
+// ranking is in fact stable and repairs stay rare.  Measured on gos2m
+// (group2, ms/step): fine split 73.1 -> 66.2 with atomics; coarse scatter
+// 74.7 -> 85.6 (kept on __match_any_sync).
+int split_atomic() {
+  static const int v = [] {
+    const char *e = getenv("SG_SPLIT_ATOMIC");
+    return e ? atoi(e) : 1;
+  }();
+  return v;
+}
+
 int64_t group_chunk_pairs() { return kChunk; }
 int32_t group_max_fanout() { return kMaxFan; }
 
@@ -510,6 +604,11 @@ cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, co
 cudaError_t group_hist(const GroupArgs &g, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
+  if (g.kbin && (g.plan.nb1 & (g.plan.nb1 - 1)) == 0) {
+    hist_bytes_kernel<<<(unsigned)((g.plan.nchunks + kHistChunks - 1) / kHistChunks), kHThreads, 0, st>>>(g);
+    ++g_launches;
+    return cudaGetLastError();
+  }
   hist_kernel<<<(unsigned)((g.plan.nchunks + kHistChunks - 1) / kHistChunks), kHThreads, 0, st>>>(g);
   ++g_launches;
   return cudaGetLastError();
@@ -551,13 +650,17 @@ cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
   const bool c8 = g.plan.nb1 == kMaxFan;
-  const void *fn = c8 ? (const void *)scatter_kernel<true> : (const void *)scatter_kernel<false>;
+  const bool at = split_atomic() >= 2;
+  const void *fn = c8 ? (at ? (const void *)scatter_kernel<true, true> : (const void *)scatter_kernel<true, false>)
+                      : (at ? (const void *)scatter_kernel<false, true> : (const void *)scatter_kernel<false, false>);
   int per_sm = 1;
   cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
   const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, g.plan.nchunks);
-  if (c8) scatter_kernel<true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else scatter_kernel<false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  if (c8 && at) scatter_kernel<true, true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else if (c8) scatter_kernel<true, false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else if (at) scatter_kernel<false, true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else scatter_kernel<false, false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }
@@ -567,12 +670,16 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
   if (g.plan.bits - g.plan.bits1 > kMaxBits - kCoarseBits) return cudaErrorInvalidValue;
   const bool f8 = g.plan.bits == 16 && g.plan.bits1 == kCoarseBits;
-  const void *fn = f8 ? (const void *)scatter2_kernel<true> : (const void *)scatter2_kernel<false>;
+  const bool at = split_atomic() >= 1;
+  const void *fn = f8 ? (at ? (const void *)scatter2_kernel<true, true> : (const void *)scatter2_kernel<true, false>)
+                      : (at ? (const void *)scatter2_kernel<false, true> : (const void *)scatter2_kernel<false, false>);
   int per_sm = 1;
   cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
-  if (f8) scatter2_kernel<true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else scatter2_kernel<false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  if (f8 && at) scatter2_kernel<true, true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else if (f8) scatter2_kernel<true, false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else if (at) scatter2_kernel<false, true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  else scatter2_kernel<false, false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
   ++g_launches;
   return cudaGetLastError();
 }

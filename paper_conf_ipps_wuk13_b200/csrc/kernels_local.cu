@@ -1,26 +1,32 @@
 // kernels_local.cu — sort inside one key bucket and run-length segmentation:
 // the second half of the per-trial grouping (AMB-5).
 //
-// The partition (kernels_group.cu) is stable, so inside a bucket the pairs
-// of one trial are still in generator order and a STABLE sort by key alone
-// yields the canonical (key, member) order.
+// The partition (kernels_group.cu) is stable in practice, so inside a bucket
+// the pairs of one trial are in generator order and a stable sort by key
+// alone yields the canonical (key, member) order.  The warp tier (default)
+// and the CTA tier verify the full (key, member) order while writing and
+// re-sort every violating run by (key, member), so the result is canonical
+// whatever order the partition delivered.
 //
 // Three tiers by bucket size n (mean ~600 pairs):
 //  * warp_local_kernel (n <= 1024): one warp per bucket, no block barriers.
 //    One sweep over the bucket's keys stores the 20 key bits after the
 //    bucket bits in the warp's shared-memory slice and builds both 10-bit
-//    digit histograms (packed 16-bit shared atomics); two stable placement
-//    passes (LSD; __match_any_sync peers, warp-private cursors) sort an index
-//    permutation; members are gathered through L1 and written in order
-//    (coalesced) with one head bit per group start.  The rare runs where
-//    distinct keys share the 20 bits out of order are detected while writing
-//    and get a stable insertion sort by key and a second write.  Larger
-//    buckets are appended to the mid / big lists.
+//    digit histograms (packed 16-bit shared atomics); two LSD placement
+//    passes sort an index permutation, each element taking its slot with its
+//    own returning shared atomic (no __match_any_sync; SG_LOCAL_ATOMIC=0
+//    selects the match-based stable placement); members are gathered through
+//    L1 and written in order (coalesced) with one head bit per group start.
+//    The rare equal-high-digit runs found out of (key, member) order while
+//    writing (20-bit ties, or lanes served out of order) are re-sorted by
+//    (key, member) and written again.  Larger buckets are appended to the
+//    mid / big lists.
 //  * local_kernel (n <= 4096, mid list): the same passes by a 256-thread CTA.
 //  * big_kernel (n > 4096, big list; groups of huge cliques): one CTA per
 //    bucket, bitonic sort by (key, member) in global (L2-resident) memory.
 // The mid and big tiers read their list lengths on the device (no host sync).
 #include <algorithm>
+#include <cstdlib>
 
 #include "group_common.cuh"
 #include "kernels.h"
@@ -118,12 +124,35 @@ __device__ __forceinline__ void warp_scan_1024(uint16_t *cnt) {
 // batch (__match_any_sync, converged with the full mask; invalid lanes carry
 // the sentinel digit kWDigits); the lowest peer advances the packed-u16
 // cursor with a returning shared atomic, four batches in flight.
-template <bool FIRST>
+// ATOMIC: every element takes its slot with its own returning shared atomic
+// (no __match_any_sync: its latency headed the kernel's stall list).  The
+// order of same-address atomics within one warp instruction is not
+// specified, so the placement may be unstable; warp_emit then verifies the
+// full (key, member) order and the caller re-sorts the violating runs.
+template <bool FIRST, bool ATOMIC>
 __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint16_t *src,
                                            uint16_t *cur, uint16_t *dst, int shift) {
   const int lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   uint32_t *cw = reinterpret_cast<uint32_t *>(cur);
+  if (ATOMIC) {
+    for (int i0 = 0; i0 < n; i0 += 32 * kWB) {
+      uint32_t e[kWB], d[kWB], o[kWB];
+#pragma unroll
+      for (int u = 0; u < kWB; ++u) {
+        const int i = i0 + u * 32 + lane;
+        const bool valid = i < n;
+        e[u] = valid ? (FIRST ? (uint32_t)i : (uint32_t)src[i]) : 0u;
+        d[u] = valid ? (S.d20[e[u]] >> shift) & (kWDigits - 1) : 0u;
+        o[u] = valid ? atomicAdd(&cw[d[u] >> 1], 1u << ((d[u] & 1) << 4)) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < kWB; ++u)
+        if (i0 + u * 32 + lane < n) dst[(o[u] >> ((d[u] & 1) << 4)) & 0xFFFFu] = (uint16_t)e[u];
+    }
+    __syncwarp();
+    return;
+  }
   for (int i0 = 0; i0 < n; i0 += 32 * kWB) {
     uint32_t e[kWB], d[kWB], m[kWB], o[kWB];
 #pragma unroll
@@ -150,14 +179,17 @@ __device__ __forceinline__ void warp_place(const WarpSmem &S, int n, const uint1
 }
 
 // Write members (and sorted keys) in the order pm; head bits into S.hb.
-// Returns true if some adjacent pair is out of key order (a 20-bit tie).
+// Returns true if some adjacent pair is out of key order (a 20-bit tie), or,
+// with FULL, out of (key, member) order.
 // Gathers of four batches are issued before their stores.
+template <bool FULL>
 __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n,
                                           const uint16_t *pm, const uint64_t *__restrict__ Kg,
                                           const uint32_t *__restrict__ Vg, int64_t gbase) {
   const int lane = threadIdx.x & 31;
   bool bad = false;
   uint64_t carry = 0;
+  uint32_t carryv = 0;
   for (int p0 = 0; p0 < n; p0 += 32 * kWB) {
     int e[kWB];
     uint64_t ke[kWB];
@@ -181,12 +213,18 @@ __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n
       uint64_t prev = __shfl_up_sync(0xffffffffu, ke[u], 1);
       if (lane == 0) prev = carry;
       carry = __shfl_sync(0xffffffffu, ke[u], 31);
+      uint32_t prevv = 0;
+      if (FULL) {
+        prevv = __shfl_up_sync(0xffffffffu, ve[u], 1);
+        if (lane == 0) prevv = carryv;
+        carryv = __shfl_sync(0xffffffffu, ve[u], 31);
+      }
       bool head = false;
       if (valid) {
         g.members[gbase + p] = ve[u];
         if (g.okeys) g.okeys[gbase + p] = ke[u];
         head = (p == 0) || prev != ke[u];
-        bad |= (p > 0) && ke[u] < prev;
+        bad |= (p > 0) && (ke[u] < prev || (FULL && ke[u] == prev && ve[u] < prevv));
       }
       const uint32_t hw = __ballot_sync(0xffffffffu, head);
       if (lane == 0) S.hb[(p0 >> 5) + u] = hw;
@@ -197,7 +235,8 @@ __device__ __forceinline__ bool warp_emit(const GroupArgs &g, WarpSmem &S, int n
 
 // BITS > 0: the plan's bucket bits known at compile time (16: the level-II
 // plans of the 2M / 640M configs), so the sort digits are constant shifts.
-template <int BITS>
+// ATOMIC: atomic (possibly unstable) placements + full-order verification.
+template <int BITS, bool ATOMIC>
 __global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
@@ -258,11 +297,48 @@ __global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __gri
     warp_scan_1024(S.cA);
     warp_scan_1024(S.cB);
     __syncwarp();
-    warp_place<true>(S, n, nullptr, S.cA, S.pa, 0);
+    warp_place<true, ATOMIC>(S, n, nullptr, S.cA, S.pa, 0);
     uint16_t *pm = S.cA;                    // the low-digit cursors are spent
-    warp_place<false>(S, n, S.pa, S.cB, pm, kWDigitBits);
+    warp_place<false, ATOMIC>(S, n, S.pa, S.cB, pm, kWDigitBits);
     const int64_t gbase = obase + sb;
-    if (warp_emit(g, S, n, pm, Kg, Vg, gbase)) {
+    if (ATOMIC && warp_emit<true>(g, S, n, pm, Kg, Vg, gbase)) {
+      // some equal-high-digit run is out of (key, member) order (an unstable
+      // atomic placement, or a 20-bit tie): re-sort each such run by (key,
+      // member) — a strict total order, so the result is canonical — and
+      // emit again
+      __syncwarp();
+      S.hb[lane] = 0;
+      __syncwarp();
+      for (int p = lane + 1; p < n; p += 32) {
+        const uint16_t ep = pm[p], eq = pm[p - 1];
+        if (pair_less(Kg[ep], Vg[ep], Kg[eq], Vg[eq])) {
+          const uint32_t dp = S.d20[ep] >> kWDigitBits;
+          int a = p - 1;
+          while (a > 0 && (S.d20[pm[a - 1]] >> kWDigitBits) == dp) --a;
+          atomicOr(&S.hb[a >> 5], 1u << (a & 31));
+        }
+      }
+      __syncwarp();
+      uint32_t word = S.hb[lane];
+      __syncwarp();
+      while (word) {
+        const int a = lane * 32 + __ffs(word) - 1;
+        word &= word - 1;
+        const uint32_t da = S.d20[pm[a]] >> kWDigitBits;
+        int b = a + 1;
+        while (b < n && (S.d20[pm[b]] >> kWDigitBits) == da) ++b;
+        for (int x = a + 1; x < b; ++x) {
+          const uint16_t e = pm[x];
+          const uint64_t ke = Kg[e];
+          const uint32_t ve = Vg[e];
+          int y = x - 1;
+          while (y >= a && pair_less(ke, ve, Kg[pm[y]], Vg[pm[y]])) { pm[y + 1] = pm[y]; --y; }
+          pm[y + 1] = e;
+        }
+      }
+      __syncwarp();
+      warp_emit<true>(g, S, n, pm, Kg, Vg, gbase);
+    } else if (!ATOMIC && warp_emit<false>(g, S, n, pm, Kg, Vg, gbase)) {
       // distinct keys sharing the 20 bits out of key order: mark the start of
       // each such equal-20-bit run, sort each run by key (stable), emit again
       __syncwarp();
@@ -295,7 +371,7 @@ __global__ void __launch_bounds__(kWWarps * 32, 3) warp_local_kernel(const __gri
         }
       }
       __syncwarp();
-      warp_emit(g, S, n, pm, Kg, Vg, gbase);
+      warp_emit<false>(g, S, n, pm, Kg, Vg, gbase);
     }
     __syncwarp();
     store_heads(g.head, S.hb, gbase, n, lane, 32);
@@ -415,9 +491,12 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
     for (int i = threadIdx.x; i < (kLocalCap / 32 + 2); i += blockDim.x) S.hb[i] = 0;
     if (threadIdx.x == 0) S.nfix = 0;
     __syncthreads();
+    // (the check and the repair use the full (key, member) order, so an
+    // input that is not in generator order — atomic split ranking — is
+    // repaired too)
     for (int p = threadIdx.x + 1; p < n; p += blockDim.x) {
       const uint64_t kp = K[pm[p]];
-      if (kp < K[pm[p - 1]]) {
+      if (pair_less(kp, S.V[pm[p]], K[pm[p - 1]], S.V[pm[p - 1]])) {
         const uint32_t dp = d16(kp);
         int a = p - 1;
         while (a > 0 && d16(K[pm[a - 1]]) == dp) --a;
@@ -437,8 +516,9 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
         for (int x = 1; x < n; ++x) {
           const uint16_t e = q2[x];
           const uint64_t ke = K[e];
+          const uint32_t ve = S.V[e];
           int y = x - 1;
-          while (y >= 0 && ke < K[q2[y]]) { q2[y + 1] = q2[y]; --y; }
+          while (y >= 0 && pair_less(ke, ve, K[q2[y]], S.V[q2[y]])) { q2[y + 1] = q2[y]; --y; }
           q2[y + 1] = e;
         }
       }
@@ -451,8 +531,9 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
       for (int x = a + 1; x < b; ++x) {
         const uint16_t e = q2[x];
         const uint64_t ke = K[e];
+        const uint32_t ve = S.V[e];
         int y = x - 1;
-        while (y >= a && ke < K[q2[y]]) { q2[y + 1] = q2[y]; --y; }   // strict: stable
+        while (y >= a && pair_less(ke, ve, K[q2[y]], S.V[q2[y]])) { q2[y + 1] = q2[y]; --y; }
         q2[y + 1] = e;
       }
     }
@@ -536,7 +617,16 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   {
     const size_t smem = sizeof(WarpSmem) * kWWarps;
     const bool b16 = g.plan.bits == 16;
-    const void *fn = b16 ? (const void *)warp_local_kernel<16> : (const void *)warp_local_kernel<0>;
+    // default: atomic placements + full-order verification (SG_LOCAL_ATOMIC=0:
+    // the match-based stable placements, key-only tie check)
+    // (forced on when the splits rank atomically: only the verifying tier
+    // repairs members that arrive out of generator order)
+    static const bool atom = [] {
+      const char *e = getenv("SG_LOCAL_ATOMIC");
+      return !(e && atoi(e) == 0) || split_atomic() > 0;
+    }();
+    const void *fn = b16 ? (atom ? (const void *)warp_local_kernel<16, true> : (const void *)warp_local_kernel<16, false>)
+                         : (atom ? (const void *)warp_local_kernel<0, true> : (const void *)warp_local_kernel<0, false>);
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
@@ -545,8 +635,10 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
     per_sm = std::max(per_sm, 1);
     const int64_t want = (nq + kWWarps - 1) / kWWarps;
     const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, want);
-    if (b16) warp_local_kernel<16><<<grid, kWWarps * 32, smem, st>>>(g);
-    else warp_local_kernel<0><<<grid, kWWarps * 32, smem, st>>>(g);
+    if (b16 && atom) warp_local_kernel<16, true><<<grid, kWWarps * 32, smem, st>>>(g);
+    else if (b16) warp_local_kernel<16, false><<<grid, kWWarps * 32, smem, st>>>(g);
+    else if (atom) warp_local_kernel<0, true><<<grid, kWWarps * 32, smem, st>>>(g);
+    else warp_local_kernel<0, false><<<grid, kWWarps * 32, smem, st>>>(g);
     ++g_launches;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }

@@ -265,8 +265,11 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
 #pragma unroll
               for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
             }
-            if (part == 0)
-              a.keys[(int64_t)j * a.key_stride + r0 + rr] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+            if (part == 0) {
+              const uint64_t key = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+              a.keys[(int64_t)j * a.key_stride + r0 + rr] = key;
+              if (a.kbin) a.kbin[(int64_t)j * a.key_stride + r0 + rr] = (uint8_t)(key >> 56);
+            }
           }
         }
         continue;
@@ -367,9 +370,27 @@ __global__ void __launch_bounds__(kMhThreads, 4) minhash_tile_kernel(const __gri
                                               2 * pp) = make_ulonglong2(k0, k1);
             }
           }
+          if (a.kbin && lane < T) {
+            // the tile's TR top key bytes of trial `lane`: one TR-byte store
+            const uint32_t *hi = reinterpret_cast<const uint32_t *>(sOut);
+            uint32_t w[TR / 4];
+#pragma unroll
+            for (int q = 0; q < TR / 4; ++q) {
+              w[q] = 0;
+#pragma unroll
+              for (int x = 0; x < 4; ++x)
+                w[q] |= (hi[2 * out_slot(4 * q + x, lane) + 1] >> 24) << (8 * x);
+            }
+            uint8_t *bd = a.kbin + (int64_t)(tp.t0 + lane) * a.key_stride + r0;
+            if (TR == 16) *reinterpret_cast<uint4 *>(bd) = make_uint4(w[0], w[1], w[2], w[3]);
+            else *reinterpret_cast<uint2 *>(bd) = make_uint2(w[0], w[1]);
+          }
         } else if (part == 0) {
           uint64_t *dst = a.keys + (int64_t)j * a.key_stride + r0;
           for (int rr = 0; rr < nr; ++rr) dst[rr] = sOut[out_slot(rr, tl)];
+          if (a.kbin)
+            for (int rr = 0; rr < nr; ++rr)
+              a.kbin[(int64_t)j * a.key_stride + r0 + rr] = (uint8_t)(sOut[out_slot(rr, tl)] >> 56);
         }
         __syncwarp();
       }
@@ -470,7 +491,9 @@ __global__ void __launch_bounds__(kMhThreads) hub_kernel(const __grid_constant__
           for (int x = 1; x < kMhWarps; ++x)
 #pragma unroll
             for (int i = 0; i < S; ++i) insert_min<S>(m, sPart[x][lane][i]);
-          a.keys[(int64_t)j * a.key_stride + row] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+          const uint64_t key = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+          a.keys[(int64_t)j * a.key_stride + row] = key;
+          if (a.kbin) a.kbin[(int64_t)j * a.key_stride + row] = (uint8_t)(key >> 56);
         }
         __syncthreads();
       }

@@ -81,6 +81,7 @@ struct KeyChunk {
   int32_t t0 = 0, nt = 0;
   bool computed = false;
   DBuf keys;
+  DBuf kbin;                       // top key bytes (single rank, grouping v1), or empty
   DBuf ctr;                        // the min-hash tile counters (kept while in flight)
   cudaEvent_t done = nullptr;      // recorded on the side stream when computed there
 };
@@ -151,6 +152,7 @@ struct sg_graph {
   cudaStream_t side = nullptr;     // min-hash of later trial chunks, overlapped with grouping
   int32_t rank = 0, world = 1;
   sg::Exchange *xch = nullptr;      // owner-routed exchange path (world > 1, or SG_DIST_EXCHANGE)
+  bool peer_xch = false;            // SG_DIST_PEER: fused exchange over peer memory
   cudaMemPool_t pool = nullptr;     // the handle's private stream-ordered pool
   int num_sms = 148;
   // graph (global n; this rank's rows [row_lo, row_hi))

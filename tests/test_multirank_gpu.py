@@ -24,7 +24,7 @@ def B():
     return binding
 
 
-def run_ranks(B, g, world, s1, c1, seed1, s2, c2, seed2, env_budget=None):
+def run_ranks(B, g, world, s1, c1, seed1, s2, c2, seed2, env_budget=None, peer=False):
     lb = B.sg_loopback_create(world)
     res, errs = [None] * world, [None] * world
 
@@ -32,7 +32,8 @@ def run_ranks(B, g, world, s1, c1, seed1, s2, c2, seed2, env_budget=None):
         h = None
         try:
             h = B.shingle_graph_create(g.row_ptr, g.col,
-                                       dist={"rank": r, "world": world, "device": 0, "loopback": lb})
+                                       dist={"rank": r, "world": world, "device": 0, "loopback": lb,
+                                             "peer": peer})
             B.shingle_pass(h, s1, c1, seed1)
             B.group_by_shingle(h)
             B.shingle_pass(h, s2, c2, seed2)
@@ -165,6 +166,36 @@ def test_loopback_big_bucket_and_empty_rank(B):
     res = run_ranks(B, g, 2, 2, 10, 1, 2, 10, 2)
     ref = oracle.shingling(g.row_ptr, g.col, 2, 10, 1, 2, 10, 2)
     check(res, ref, 10, 10)
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("world,s1,c1,s2,c2", [(2, 2, 100, 2, 100), (3, 3, 33, 3, 31),
+                                               (4, 2, 64, 8, 3), (5, 4, 40, 1, 64)])
+def test_loopback_fused_peer_exchange(B, world, s1, c1, s2, c2):
+    """SG_DIST_PEER: the owner-partition kernel stores every
+    pair straight into its owner's receive buffer (peer pointers of the other
+    virtual ranks); no send buffer, no send / recv.  Same outputs as the
+    oracle, element by element."""
+    g = SG.make("tiny")
+    res = run_ranks(B, g, world, s1, c1, 1000 + c1, s2, c2, 2000 + c2, peer=True)
+    ref = oracle.shingling(g.row_ptr, g.col, s1, c1, 1000 + c1, s2, c2, 2000 + c2)
+    check(res, ref, c1, c2)
+
+
+@pytest.mark.timeout(900)
+def test_loopback_fused_peer_small_and_chunked(B, monkeypatch):
+    """The fused exchange on the homology-shaped `small` config, once with
+    the planner forced into several trial chunks (the receive buffers are
+    reused chunk after chunk behind the per-chunk barriers)."""
+    g = SG.make("small")
+    cfg = SG.CONFIGS["small"]
+    args = (cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"])
+    ref = oracle.shingling(g.row_ptr, g.col, *args)
+    check(run_ranks(B, g, 2, *args, peer=True), ref, cfg["c1"], cfg["c2"])
+    monkeypatch.setenv("SG_MEM_BUDGET", str(150 << 20))   # level II in several trial chunks
+    res = run_ranks(B, g, 3, *args, peer=True)
+    check(res, ref, cfg["c1"], cfg["c2"])
+    assert any(abs(r["counts"]["chunks1"]) > 1 or abs(r["counts"]["chunks2"]) > 1 for r in res)
 
 
 @pytest.mark.timeout(300)

@@ -65,6 +65,23 @@ def test_nccl_world1_exchange_path(B):
             B.shingle_graph_destroy(h)
 
 
+@pytest.mark.timeout(600)
+def test_nccl_world1_fused_peer_exchange(B):
+    """SG_DIST_PEER on a one-rank NCCL communicator: the receive buffers are
+    published over the communicator (ncclAllGather), the owner-partition
+    kernel stores into them, the barriers are NCCL all-gathers."""
+    g = SG.make("tiny")
+    args = (2, 37, 101, 2, 33, 102)
+    ref = oracle.shingling(g.row_ptr, g.col, *args)
+    uid = B.nccl_unique_id()
+    h = B.shingle_graph_create(g.row_ptr, g.col,
+                               dist=dict(rank=0, world=1, device=0, nccl_uid=uid, exchange=True, peer=True))
+    try:
+        check(run_exchange(B, h, g, args), ref)
+    finally:
+        B.shingle_graph_destroy(h)
+
+
 def test_load_replaces_the_graph_and_rejects_bad_csr(B):
     g = SG.make("tiny")
     args = (2, 9, 101, 2, 7, 102)
