@@ -260,16 +260,21 @@ __global__ void __launch_bounds__(kHThreads) hist_kernel(const __grid_constant__
 }
 
 // The same histogram from the min-hash kernels' top-key-byte array (1 B per
-// pair instead of the 8-B key; power-of-two coarse fan-outs of <= 256 bins):
-// one 4-byte load per thread and chunk.
+// pair instead of the 8-B key; power-of-two coarse fan-outs of <= 256 bins).
+// A chunk is 4 KB, one 4-byte word per thread: chunks are counted four at a
+// time (four words in flight per thread, the next four prefetched), else the
+// kernel is latency bound on too few bytes in flight.
+constexpr int kHB = 4;                         // chunks counted together
+template <bool B8>                             // B8: nb1 == 256 (the bin is the byte)
 __global__ void __launch_bounds__(kHThreads) hist_bytes_kernel(const __grid_constant__ GroupArgs g) {
-  __shared__ uint32_t hist[kMaxFan];
-  const int nb = (int)g.plan.nb1;
-  const int sh = 8 - grp::bits_for(nb);
+  __shared__ uint32_t hist[kHB][kMaxFan];
+  const int nb = B8 ? kMaxFan : (int)g.plan.nb1;
+  const int sh = B8 ? 0 : 8 - grp::bits_for(nb);
   const int64_t k0 = (int64_t)blockIdx.x * kHistChunks;
   const int64_t k1 = min(k0 + kHistChunks, g.plan.nchunks);
-  for (int i = threadIdx.x; i < kMaxFan; i += kHThreads) hist[i] = 0;
+  for (int i = threadIdx.x; i < kHB * kMaxFan; i += kHThreads) (&hist[0][0])[i] = 0;
   auto load = [&](int64_t k) -> uint32_t {
+    if (k >= k1) return 0u;
     const int len = g.plan.chunk_len[k];
     const uint8_t *__restrict__ kb = g.kbin + g.plan.chunk_in0[k];
     const int i = 4 * threadIdx.x;
@@ -278,22 +283,35 @@ __global__ void __launch_bounds__(kHThreads) hist_bytes_kernel(const __grid_cons
     for (int x = 0; x < 4 && i + x < len; ++x) w |= (uint32_t)kb[i + x] << (8 * x);
     return w;
   };
-  uint32_t cur = k0 < k1 ? load(k0) : 0u;
-  __syncthreads();
-  for (int64_t k = k0; k < k1; ++k) {
-    const uint32_t nxt = k + 1 < k1 ? load(k + 1) : 0u;   // in flight while counting
-    const int len = g.plan.chunk_len[k];
+  uint32_t cur[kHB], nxt[kHB];
 #pragma unroll
-    for (int x = 0; x < 4; ++x)
-      if (4 * (int)threadIdx.x + x < len) atomicAdd(&hist[((cur >> (8 * x)) & 0xFFu) >> sh], 1u);
-    __syncthreads();
-    uint32_t *out = g.counts + k * nb;
-    for (int i = threadIdx.x; i < nb; i += kHThreads) {
-      out[i] = hist[i];
-      hist[i] = 0;
+  for (int c = 0; c < kHB; ++c) cur[c] = load(k0 + c);
+  __syncthreads();
+  for (int64_t kb0 = k0; kb0 < k1; kb0 += kHB) {
+#pragma unroll
+    for (int c = 0; c < kHB; ++c) nxt[c] = load(kb0 + kHB + c);   // in flight while counting
+#pragma unroll
+    for (int c = 0; c < kHB; ++c) {
+      if (kb0 + c >= k1) break;
+      const int len = g.plan.chunk_len[kb0 + c];
+      if (len == kChunk) {                     // warp-uniform: whole chunk, no tail tests
+#pragma unroll
+        for (int x = 0; x < 4; ++x) atomicAdd(&hist[c][((cur[c] >> (8 * x)) & 0xFFu) >> sh], 1u);
+      } else {
+#pragma unroll
+        for (int x = 0; x < 4; ++x)
+          if (4 * (int)threadIdx.x + x < len) atomicAdd(&hist[c][((cur[c] >> (8 * x)) & 0xFFu) >> sh], 1u);
+      }
     }
     __syncthreads();
-    cur = nxt;
+    for (int i = threadIdx.x; i < kHB * nb; i += kHThreads) {
+      const int c = i / nb, b = i - c * nb;
+      if (kb0 + c < k1) g.counts[(kb0 + c) * nb + b] = hist[c][b];
+      hist[c][b] = 0;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int c = 0; c < kHB; ++c) cur[c] = nxt[c];
   }
 }
 
@@ -310,7 +328,7 @@ __global__ void __launch_bounds__(1024) colscan_kernel(const __grid_constant__ G
   const int k0 = g.plan.trial_chunk0[j], k1 = g.plan.trial_chunk0[j + 1];
   const int L = (k1 - k0 + 31) / 32;
   const int a0 = min(k1, k0 + pi * L), a1 = min(k1, a0 + L);
-  constexpr int U = 8;                     // loads in flight per thread
+  constexpr int U = 16;                    // loads in flight per thread (latency bound)
   uint32_t s = 0;
   if (b < nb) {
     int k = a0;
@@ -605,7 +623,9 @@ cudaError_t group_hist(const GroupArgs &g, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
   if (g.kbin && (g.plan.nb1 & (g.plan.nb1 - 1)) == 0) {
-    hist_bytes_kernel<<<(unsigned)((g.plan.nchunks + kHistChunks - 1) / kHistChunks), kHThreads, 0, st>>>(g);
+    const unsigned grid = (unsigned)((g.plan.nchunks + kHistChunks - 1) / kHistChunks);
+    if (g.plan.nb1 == kMaxFan) hist_bytes_kernel<true><<<grid, kHThreads, 0, st>>>(g);
+    else hist_bytes_kernel<false><<<grid, kHThreads, 0, st>>>(g);
     ++g_launches;
     return cudaGetLastError();
   }

@@ -142,6 +142,8 @@ __device__ __forceinline__ uint32_t hash_or_pad(uint32_t A, uint32_t B, uint32_t
 
 // Two rows of na / nb (<= 4, warp-uniform) padded pairs, scanned side by
 // side: 64-bit broadcast loads, so a 2-entry row hashes 2 slots, not 4.
+// (Hashing the odd entry alone instead of testing for the padding word was
+// measured slower: 11.05e9 vs 10.87e9 instructions per 64-trial chunk.)
 template <int S>
 __device__ __forceinline__ void pairs2(const uint32_t *pa, const uint32_t *pb, int na, int nb,
                                        uint32_t A, uint32_t B, uint32_t (&ma)[S], uint32_t (&mb)[S]) {
