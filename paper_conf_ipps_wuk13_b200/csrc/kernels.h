@@ -135,7 +135,8 @@ cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, c
                          int32_t c, cudaStream_t st);
 
 int64_t group_local_capacity();
-int split_atomic();              // SG_SPLIT_ATOMIC: atomic split ranking (1: fine split, 2: + coarse)
+int split_mode(bool fine);        // ranking mode of the split kernels (SG_SPLIT_FINE / _COARSE)
+int split_atomic();              // a split may deliver pairs out of generator order
 int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
 int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
 // Bucket plan for trial segments of at most `maxseg` pairs.
@@ -172,49 +173,6 @@ cudaError_t group_c_bucket(const GroupArgs &g, int num_sms, cudaStream_t st);   
 // Sort the members of every listed segment ascending (count read on the device).
 cudaError_t group_c_segsort(const GroupArgs &g, int num_sms, cudaStream_t st);
 cudaError_t group_binscan(const GroupArgs &g, cudaStream_t st);   // bstart1 = scan of bsize1 per trial
-
-// ---- multi-rank helpers (kernels_pass.cu) ----------------------------------
-// counts[j] = number of rows whose rstart lies in [seg[j], seg[j+1]) (zeroed by caller)
-cudaError_t rows_per_trial(const int64_t *rstart, int64_t nrows, const int64_t *seg, int32_t c,
-                           unsigned long long *counts, cudaStream_t st);
-// rowid[i] = i + off[j] for the trial j with first[j] <= i < first[j+1]
-cudaError_t assign_rowid(uint32_t *rowid, int64_t nrows, const int64_t *first, const int64_t *off,
-                         int32_t c, cudaStream_t st);
-
-int64_t group_local_capacity();
-int split_atomic();              // SG_SPLIT_ATOMIC: atomic split ranking (1: fine split, 2: + coarse)
-int64_t group_chunk_pairs();     // pairs per partition chunk (hist and scatter)
-int32_t group_max_fanout();      // bins of one split pass (owner ranks <= this)
-// Bucket plan for trial segments of at most `maxseg` pairs.
-void group_bits(int64_t maxseg, int32_t *bits, int32_t *bits1);
-// Fill plan.chunk_* (plan.nchunks entries) from the piece table (device
-// pointers; pieces ordered by trial, chunks of group_chunk_pairs() pairs).
-cudaError_t group_chunk_tables(const GroupPlan &plan, const int32_t *p_trial, const int64_t *p_in0,
-                               const int64_t *p_len, const int64_t *p_row0,
-                               const int64_t *p_chunk0, int32_t npieces, cudaStream_t st);
-cudaError_t group_hist(const GroupArgs &g, cudaStream_t st);
-cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st);
-cudaError_t group_colscan(const GroupArgs &g, cudaStream_t st);   // chunk prefixes + bsize1 only
-cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
-cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st);   // two-level plans only
-// Sort every final bucket and write members + head bits: warp tier, then the
-// mid and big tiers over the lists the warp tier filled (no host sync).
-cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st);
-// Global-memory sort of the buckets listed in big_list (count on the device).
-cudaError_t group_big(const GroupArgs &g, int num_sms, cudaStream_t st);
-
-// ---- grouping v2 (kernels_sort.cu): one stable partition by
-// the top `plan.bits` (<= 13) key bits over super-chunks of
-// group_b_super_pairs() pairs (plan.chunk), then a shared-memory sort per
-// bucket.  Single level: plan.nbins = plan.nb1 = 2^bits, bkeys = akeys,
-// bvals = avals, bstart = bstart1, bsize = bsize1.
-int64_t group_b_super_pairs();
-int32_t group_b_max_bits();
-int32_t group_b_local_cap();
-void group_b_bits(int64_t maxseg, int32_t *bits);
-cudaError_t group_b_hist(const GroupArgs &g, cudaStream_t st);       // + offsets
-cudaError_t group_b_scatter(const GroupArgs &g, int num_sms, cudaStream_t st);
-cudaError_t group_b_local(const GroupArgs &g, int num_sms, cudaStream_t st);   // + big
 
 // ---- Phase III on the device (kernels_report.cu) ---------------------------
 struct ReportArgs {

@@ -96,13 +96,20 @@ struct SplitSmem {
 // BALLOT: peer masks from ballots (measured faster for the fine split,
 // slower for the coarse scatter) or __match_any_sync.  NBC > 0: nb == NBC is
 // known at compile time (full 8-bit fan-out: unrolled ballots, constant loops).
-// AT: no peer masks at all — every pair counts and takes its slot with its
-// own shared atomic on the warp's packed u16 counters.  Pairs of one warp
-// are visited batch by batch in input order; within one warp instruction the
-// order of conflicting lanes is the hardware's (tools/atom_order.cu measures
-// it).  The final sorts verify the full (key, member) order and repair any
-// run that is out of it, so the result never depends on that order.
-template <bool BALLOT, int NBC, bool AT, typename BIN, typename OBASE>
+// AT selects how a warp ranks its pairs:
+//  0: peer masks (__match_any_sync or ballots) for both the count and the
+//     placement, warp counters advanced by the lowest peer (stable);
+//  1: no peer masks — every pair counts and takes its slot with its own
+//     shared atomic on the warp's packed u16 counters.  Within one warp
+//     instruction the order of conflicting lanes is the hardware's
+//     (tools/atom_order.cu measures lane order on the B200); the final sorts
+//     verify the full (key, member) order and repair any run out of it, so
+//     the result never depends on it;
+//  2: counts by fire-and-forget atomics (no dependency chain), placement by
+//     peer masks as in 0 (stable);
+//  3: counts as in 2, placement by peer masks with the lowest peer taking
+//     the run's base by a returning atomic (no __syncwarp chain; stable).
+template <bool BALLOT, int NBC, int AT, typename BIN, typename OBASE>
 __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
@@ -116,7 +123,7 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
   __syncwarp();
   uint32_t pr[kPerLane];
   const int nbits = NBC > 0 ? grp::bits_for(NBC) : grp::bits_for(nb);
-  if (AT) {
+  if (AT >= 1) {
 #pragma unroll
     for (int u = 0; u < kPerLane; ++u)
       if (elem_of(u) < len) {
@@ -161,7 +168,43 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
     if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
   __syncthreads();
-  if (AT) {
+  if (AT >= 2) {
+    // peer masks of all batches first (independent, their latencies overlap)
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u) {
+      const bool valid = elem_of(u) < len;
+      const uint32_t vm = __ballot_sync(0xffffffffu, valid);
+      const uint32_t b = valid ? bin_of(kk[u]) : 0u;
+      uint32_t pm = 0;
+      if (BALLOT) pm = grp::peers_by_ballot(b, vm, nbits);
+      else if (valid) pm = __match_any_sync(vm, b);
+      pr[u] = valid ? pm : 0u;
+    }
+  }
+  if (AT == 3) {
+    uint32_t o[kPerLane];
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u) {
+      o[u] = 0;
+      if (elem_of(u) < len && (pr[u] & lt) == 0) {
+        const int idx = w * nb + (int)bin_of(kk[u]);
+        o[u] = atomicAdd(cw + (idx >> 1), (uint32_t)__popc(pr[u]) << ((idx & 1) << 4)) >> ((idx & 1) << 4);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kPerLane; ++u) {
+      const int lead = __ffs(pr[u]) - 1;
+      const uint32_t oo = __shfl_sync(0xffffffffu, o[u], lead < 0 ? 0 : lead);
+      if (elem_of(u) < len) {
+        const uint32_t p = (oo & 0xFFFFu) + __popc(pr[u] & lt);
+        S.K[p] = kk[u];
+        S.V[p] = vv[u];
+      }
+    }
+    __syncthreads();
+    return;
+  }
+  if (AT == 1) {
     uint32_t o[kPerLane];
 #pragma unroll
     for (int u = 0; u < kPerLane; ++u) {
@@ -411,7 +454,7 @@ __device__ __forceinline__ void load_chunk(const GroupArgs &g, int64_t k, uint64
 
 // C8: the full 8-bit coarse fan-out (nb1 == 256), bin = the top key byte
 // (a constant shift; the generic bin costs ~10 instructions per use).
-template <bool C8, bool AT>
+template <bool C8, int AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -457,7 +500,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
 // ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
 // F8: bits == 16 with an 8-bit coarse level (the level-II plans of the 2M and
 // 640M configs): fine digit = key bits 48..55 by a constant shift.
-template <bool F8, bool AT>
+template <bool F8, int AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -575,22 +618,27 @@ __global__ void sum_i32_kernel(const int32_t *__restrict__ a, int64_t n, unsigne
 
 }  // namespace
 
-// Ranking by per-pair shared atomics (split_place<..., AT = true>) in the
-// fine split (default; SG_SPLIT_ATOMIC=0: ballot-built peer masks) and, with
-// SG_SPLIT_ATOMIC=2, in the coarse scatter as well.  The local sorts verify
-// and repair the (key, member) order, so the outputs are the same either
-// way; on the B200 conflicting lanes are served in lane order
-// (tools/atom_order.cu: 0 of 1.55e8 warp-instructions out of order), so the
-// ranking is in fact stable and repairs stay rare.  Measured on gos2m
-// (group2, ms/step): fine split 73.1 -> 66.2 with atomics; coarse scatter
-// 74.7 -> 85.6 (kept on __match_any_sync).
-int split_atomic() {
-  static const int v = [] {
-    const char *e = getenv("SG_SPLIT_ATOMIC");
-    return e ? atoi(e) : 1;
-  }();
-  return v;
+// Ranking mode of the split kernels (split_place's AT): the fine split
+// defaults to 1 (per-pair atomics), the coarse scatter to 0 (__match_any_sync);
+// SG_SPLIT_FINE / SG_SPLIT_COARSE = 0..3 select another (A/B).  Measured on
+// gos2m (group2, ms/step): fine split 73.1 (0) -> 66.2 (1); coarse scatter
+// 74.7 (0) vs 85.6 (1).  On the B200 conflicting lanes are served in lane
+// order (tools/atom_order.cu: 0 of 1.55e8 warp-instructions out of order), so
+// mode 1 is in fact stable and the local sorts' repairs stay rare.
+int split_mode(bool fine) {
+  static const int m[2] = {[] {
+                             const char *e = getenv("SG_SPLIT_COARSE");
+                             return e ? std::min(3, std::max(0, atoi(e))) : 0;
+                           }(),
+                           [] {
+                             const char *e = getenv("SG_SPLIT_FINE");
+                             return e ? std::min(3, std::max(0, atoi(e))) : 1;
+                           }()};
+  return m[fine ? 1 : 0];
 }
+
+// Whether any split may deliver a bucket out of generator order (mode 1).
+int split_atomic() { return split_mode(false) == 1 || split_mode(true) == 1; }
 
 int64_t group_chunk_pairs() { return kChunk; }
 int32_t group_max_fanout() { return kMaxFan; }
@@ -670,17 +718,21 @@ cudaError_t group_scatter(const GroupArgs &g, int num_sms, cudaStream_t st) {
   if (g.plan.nchunks == 0) return cudaSuccess;
   if (g.plan.nb1 > kMaxFan) return cudaErrorInvalidValue;
   const bool c8 = g.plan.nb1 == kMaxFan;
-  const bool at = split_atomic() >= 2;
-  const void *fn = c8 ? (at ? (const void *)scatter_kernel<true, true> : (const void *)scatter_kernel<true, false>)
-                      : (at ? (const void *)scatter_kernel<false, true> : (const void *)scatter_kernel<false, false>);
+  const int mode = split_mode(false);
+  const void *fn = nullptr;
+  switch ((c8 ? 4 : 0) + mode) {
+#define SG_SC(C, M) case (C ? 4 : 0) + M: fn = (const void *)scatter_kernel<C, M>; break;
+    SG_SC(true, 0) SG_SC(true, 1) SG_SC(true, 2) SG_SC(true, 3)
+    SG_SC(false, 0) SG_SC(false, 1) SG_SC(false, 2) SG_SC(false, 3)
+#undef SG_SC
+  }
   int per_sm = 1;
   cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
   const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, g.plan.nchunks);
-  if (c8 && at) scatter_kernel<true, true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else if (c8) scatter_kernel<true, false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else if (at) scatter_kernel<false, true><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else scatter_kernel<false, false><<<grid, kSThreads, sizeof(SplitSmem), st>>>(g);
+  void *args[] = {(void *)&g};
+  e = cudaLaunchKernel(fn, dim3(grid), dim3(kSThreads), args, sizeof(SplitSmem), st);
+  if (e != cudaSuccess) return e;
   ++g_launches;
   return cudaGetLastError();
 }
@@ -690,16 +742,20 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
   if (g.plan.bits - g.plan.bits1 > kMaxBits - kCoarseBits) return cudaErrorInvalidValue;
   const bool f8 = g.plan.bits == 16 && g.plan.bits1 == kCoarseBits;
-  const bool at = split_atomic() >= 1;
-  const void *fn = f8 ? (at ? (const void *)scatter2_kernel<true, true> : (const void *)scatter2_kernel<true, false>)
-                      : (at ? (const void *)scatter2_kernel<false, true> : (const void *)scatter2_kernel<false, false>);
+  const int mode = split_mode(true);
+  const void *fn = nullptr;
+  switch ((f8 ? 4 : 0) + mode) {
+#define SG_SC(C, M) case (C ? 4 : 0) + M: fn = (const void *)scatter2_kernel<C, M>; break;
+    SG_SC(true, 0) SG_SC(true, 1) SG_SC(true, 2) SG_SC(true, 3)
+    SG_SC(false, 0) SG_SC(false, 1) SG_SC(false, 2) SG_SC(false, 3)
+#undef SG_SC
+  }
   int per_sm = 1;
   cudaError_t e = split_attr(fn, &per_sm);
   if (e != cudaSuccess) return e;
-  if (f8 && at) scatter2_kernel<true, true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else if (f8) scatter2_kernel<true, false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else if (at) scatter2_kernel<false, true><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
-  else scatter2_kernel<false, false><<<(unsigned)nq1, kSThreads, sizeof(SplitSmem), st>>>(g);
+  void *args[] = {(void *)&g};
+  e = cudaLaunchKernel(fn, dim3((unsigned)nq1), dim3(kSThreads), args, sizeof(SplitSmem), st);
+  if (e != cudaSuccess) return e;
   ++g_launches;
   return cudaGetLastError();
 }

@@ -534,11 +534,201 @@ cudaError_t launch_tile(MhParams &P, int num_sms, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// ---- pass II, windowed row-per-lane (default for 16-row-tile passes) --------
+// The tile kernel gives every (row, trial) of a ~5-entry pass-II row the
+// per-row costs of a lane = trial scan (row metadata, staging, loop control:
+// ~134 instructions per (row, trial)).  Here a CTA takes a
+// window of 256 consecutive rows and sorts them by length class in shared
+// memory; warp w takes the w-th 32 rows of that order, one row per lane,
+// with the row's <= 8 entries in registers and each trial's (A, B) a
+// shared-memory broadcast (lengths agree inside a warp except at the class
+// boundaries).  Rows of 9..kHubLen entries are taken one at a time by a
+// warp, lane = trial.  The keys of one 32-trial pass are staged in shared
+// memory ([trial][row], 64 KB) and written in natural row order: a trial's
+// 256 keys are one coalesced 2 KB store, so the output layout and the
+// generator order the stable grouping needs are unchanged.  Hub rows are
+// left to hub_kernel (launched after, its stores win).
+constexpr int kWin = 256;                      // rows per window = threads per CTA
+
+template <int S, int L, bool PAD>
+__device__ __forceinline__ uint64_t row_key(const uint32_t (&v)[8], uint32_t A, uint32_t B,
+                                            uint64_t seed, int j);
+
+template <int S, int L, bool PAD>
+__device__ __forceinline__ void win_short(const uint32_t *sA, const uint32_t *sB, const uint32_t (&v)[8],
+                                          uint64_t *sK, int lr, bool act, int tp0, int T, uint64_t seed,
+                                          int t0) {
+  for (int j = 0; j < T; ++j) {
+    const uint64_t key = row_key<S, L, PAD>(v, sA[tp0 + j], sB[tp0 + j], seed, t0 + tp0 + j);
+    if (act) sK[j * kWin + lr] = key;
+  }
+}
+
+template <int S>
+__global__ void __launch_bounds__(kWin, 3) minhash_win_kernel(const __grid_constant__ MinhashArgs a) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  uint64_t *sK = reinterpret_cast<uint64_t *>(smraw);                 // [32][kWin]
+  uint32_t *sA = reinterpret_cast<uint32_t *>(sK + 32 * kWin);
+  uint32_t *sB = sA + a.nt;
+  __shared__ uint16_t sOrd[kWin];
+  __shared__ uint32_t sCnt[12], sCur[12], sLong;
+  __shared__ int64_t sWin;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, t = threadIdx.x;
+  for (int i = t; i < a.nt; i += kWin) {
+    sA[i] = a.A[a.t0 + i];
+    sB[i] = a.B[a.t0 + i];
+  }
+  const int64_t nwin = (a.nrows + kWin - 1) / kWin;
+  for (;;) {
+    if (t == 0) sWin = (int64_t)atomicAdd(a.counter, 1ull);
+    if (t < 12) sCnt[t] = 0;
+    __syncthreads();
+    const int64_t win = sWin;
+    if (win >= nwin) break;
+    const int64_t r0 = win * kWin;
+    const int64_t r = r0 + t;
+    const int len = r < a.nrows ? a.rlen[r] : 0;
+    // class: 1..8 short (register rows), 9 long (lane = trial), 10 hub / none
+    const int cls = len == 0 ? 10 : len <= 8 ? len : len <= kHubLen ? 9 : 10;
+    atomicAdd(&sCnt[cls], 1u);
+    __syncthreads();
+    if (t == 0) {
+      uint32_t run = 0;
+      for (int c = 0; c < 12; ++c) {
+        sCur[c] = run;
+        run += sCnt[c];
+      }
+      sLong = 0;
+    }
+    __syncthreads();
+    sOrd[atomicAdd(&sCur[cls], 1u)] = (uint16_t)t;
+    __syncthreads();
+    const int nshort = (int)(sCnt[1] + sCnt[2] + sCnt[3] + sCnt[4] + sCnt[5] + sCnt[6] + sCnt[7] + sCnt[8]);
+    const int nlong = (int)sCnt[9];
+    // this lane's short row, in registers for every pass
+    const int slot = w * 32 + lane;
+    const bool act = slot < nshort;
+    const int lr = act ? sOrd[slot] : 0;
+    int rl = 0;
+    uint32_t v[8];
+    if (act) {
+      rl = a.rlen[r0 + lr];
+      const uint32_t *src = a.entries + a.rstart[r0 + lr];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] = e < rl ? src[e] : 0xFFFFFFFFu;
+    } else {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] = 0xFFFFFFFFu;
+    }
+    const bool any_short = __any_sync(0xffffffffu, act);
+    const int lw = __reduce_max_sync(0xffffffffu, (unsigned)rl);
+    const int lmin = __reduce_min_sync(0xffffffffu, act ? (unsigned)rl : 8u);
+    for (int tp0 = 0; tp0 < a.nt; tp0 += 32) {
+      const int T = min(32, a.nt - tp0);
+      if (any_short) {
+        if (lmin != lw) {
+          win_short<S, 8, true>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0);
+        } else {
+          switch (lw) {
+            case 1: win_short<S, 1, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 2: win_short<S, 2, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 3: win_short<S, 3, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 4: win_short<S, 4, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 5: win_short<S, 5, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 6: win_short<S, 6, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            case 7: win_short<S, 7, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+            default: win_short<S, 8, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
+          }
+        }
+      }
+      // long rows, one per warp at a time (dynamic), lane = trial
+      for (;;) {
+        int li = 0;
+        if (lane == 0) li = (int)atomicAdd(&sLong, 1u);
+        li = __shfl_sync(0xffffffffu, li, 0);
+        if (li >= nlong) break;
+        const int lrow = sOrd[nshort + li];
+        const int ll = a.rlen[r0 + lrow];
+        const uint32_t *src = a.entries + a.rstart[r0 + lrow];
+        const int j = tp0 + (lane < T ? lane : 0);
+        const uint32_t A = sA[j], B = sB[j];
+        uint32_t m[S];
+#pragma unroll
+        for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
+        int e = 0;
+        for (; e + 4 <= ll; e += 4) {
+          const uint32_t x0 = src[e], x1 = src[e + 1], x2 = src[e + 2], x3 = src[e + 3];
+          insert_min<S>(m, m31_hash(A, B, x0));
+          insert_min<S>(m, m31_hash(A, B, x1));
+          insert_min<S>(m, m31_hash(A, B, x2));
+          insert_min<S>(m, m31_hash(A, B, x3));
+        }
+        for (; e < ll; ++e) insert_min<S>(m, m31_hash(A, B, src[e]));
+        if (lane < T) sK[lane * kWin + lrow] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+      }
+      __syncthreads();
+      // natural-order write-out: trial j's kWin keys are contiguous
+      const int nr = (int)min((int64_t)kWin, a.nrows - r0);
+      for (int j = 0; j < T; ++j) {
+        if (t < nr) a.keys[(int64_t)(tp0 + j) * a.key_stride + r0 + t] = sK[j * kWin + t];
+      }
+      if (a.kbin) {
+        for (int idx = t; idx < T * (kWin / 4); idx += kWin) {
+          const int j = idx / (kWin / 4), q = idx % (kWin / 4);
+          if (4 * q < nr) {
+            const uint32_t *hi = reinterpret_cast<const uint32_t *>(sK + j * kWin + 4 * q);
+            const uint32_t word = (hi[1] >> 24) | ((hi[3] >> 24) << 8) | ((hi[5] >> 24) << 16) |
+                                  ((hi[7] >> 24) << 24);
+            *reinterpret_cast<uint32_t *>(a.kbin + (int64_t)(tp0 + j) * a.key_stride + r0 + 4 * q) = word;
+          }
+        }
+      }
+      __syncthreads();
+      if (t == 0) sLong = 0;
+      __syncthreads();
+    }
+  }
+}
+
+template <int S>
+cudaError_t launch_win(MhParams &P, int num_sms, cudaStream_t st) {
+  const size_t smem = (size_t)32 * kWin * 8 + (size_t)2 * P.a.nt * 4;
+  auto kern = minhash_win_kernel<S>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWin, smem);
+  if (e != cudaSuccess) return e;
+  per_sm = std::max(per_sm, 1);
+  const int64_t nwin = (P.a.nrows + kWin - 1) / kWin;
+  const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, std::max<int64_t>(nwin, 1));
+  kern<<<grid, kWin, smem, st>>>(P.a);
+  ++g_launches;
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  const size_t hsm = (size_t)kHubStage * 4;
+  if ((e = cudaFuncSetAttribute(hub_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)hsm)) != cudaSuccess)
+    return e;
+  hub_kernel<S><<<num_sms * 3, kMhThreads, hsm, st>>>(P);
+  ++g_launches;
+  return cudaGetLastError();
+}
+
 // Short rows (pass II) take 16-row tiles: a trial's keys of one tile are a
 // full 128 B line; long rows (pass I) keep 8-row tiles (the stage holds them).
+// SG_MH_TILE16=1 (A/B): the 16-row tile kernel instead of the windowed
+// row-per-lane kernel for pass II.
+static bool use_tile16() {
+  static const bool v = [] {
+    const char *e = getenv("SG_MH_TILE16");
+    return e && atoi(e) != 0;
+  }();
+  return v;
+}
+
 template <int S>
 cudaError_t launch_s(MhParams &P, int num_sms, cudaStream_t st) {
-  if (P.a.tile_rows == 16) return launch_tile<S, 16>(P, num_sms, st);
+  if (P.a.tile_rows == 16) return use_tile16() ? launch_tile<S, 16>(P, num_sms, st) : launch_win<S>(P, num_sms, st);
   return launch_tile<S, 8>(P, num_sms, st);
 }
 
