@@ -549,6 +549,7 @@ cudaError_t launch_tile(MhParams &P, int num_sms, cudaStream_t st) {
 // generator order the stable grouping needs are unchanged.  Hub rows are
 // left to hub_kernel (launched after, its stores win).
 constexpr int kWin = 256;                      // rows per window = threads per CTA
+constexpr int kWT = 16;                        // trials per staged pass (32 KB of keys)
 
 template <int S, int L, bool PAD>
 __device__ __forceinline__ uint64_t row_key(const uint32_t (&v)[8], uint32_t A, uint32_t B,
@@ -565,10 +566,10 @@ __device__ __forceinline__ void win_short(const uint32_t *sA, const uint32_t *sB
 }
 
 template <int S>
-__global__ void __launch_bounds__(kWin, 3) minhash_win_kernel(const __grid_constant__ MinhashArgs a) {
+__global__ void __launch_bounds__(kWin, 4) minhash_win_kernel(const __grid_constant__ MinhashArgs a) {
   extern __shared__ __align__(16) unsigned char smraw[];
-  uint64_t *sK = reinterpret_cast<uint64_t *>(smraw);                 // [32][kWin]
-  uint32_t *sA = reinterpret_cast<uint32_t *>(sK + 32 * kWin);
+  uint64_t *sK = reinterpret_cast<uint64_t *>(smraw);                 // [kWT][kWin]
+  uint32_t *sA = reinterpret_cast<uint32_t *>(sK + kWT * kWin);
   uint32_t *sB = sA + a.nt;
   __shared__ uint16_t sOrd[kWin];
   __shared__ uint32_t sCnt[12], sCur[12], sLong;
@@ -623,23 +624,21 @@ __global__ void __launch_bounds__(kWin, 3) minhash_win_kernel(const __grid_const
     const bool any_short = __any_sync(0xffffffffu, act);
     const int lw = __reduce_max_sync(0xffffffffu, (unsigned)rl);
     const int lmin = __reduce_min_sync(0xffffffffu, act ? (unsigned)rl : 8u);
-    for (int tp0 = 0; tp0 < a.nt; tp0 += 32) {
-      const int T = min(32, a.nt - tp0);
+    for (int tp0 = 0; tp0 < a.nt; tp0 += kWT) {
+      const int T = min(kWT, a.nt - tp0);
       if (any_short) {
-        if (lmin != lw) {
-          win_short<S, 8, true>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0);
-        } else {
-          switch (lw) {
-            case 1: win_short<S, 1, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 2: win_short<S, 2, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 3: win_short<S, 3, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 4: win_short<S, 4, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 5: win_short<S, 5, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 6: win_short<S, 6, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            case 7: win_short<S, 7, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-            default: win_short<S, 8, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0); break;
-          }
+        // the warp's longest row sets the unrolled length; only a warp that
+        // mixes lengths (a class boundary of the window order) pays the pad test
+#define SG_WS(L)                                                                          \
+  case L:                                                                                 \
+    if (lmin != lw) win_short<S, L, true>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0);  \
+    else win_short<S, L, false>(sA, sB, v, sK, lr, act, tp0, T, a.seed, a.t0);            \
+    break;
+        switch (lw) {
+          SG_WS(1) SG_WS(2) SG_WS(3) SG_WS(4) SG_WS(5) SG_WS(6) SG_WS(7)
+          default: SG_WS(8)
         }
+#undef SG_WS
       }
       // long rows, one per warp at a time (dynamic), lane = trial
       for (;;) {
@@ -650,21 +649,32 @@ __global__ void __launch_bounds__(kWin, 3) minhash_win_kernel(const __grid_const
         const int lrow = sOrd[nshort + li];
         const int ll = a.rlen[r0 + lrow];
         const uint32_t *src = a.entries + a.rstart[r0 + lrow];
-        const int j = tp0 + (lane < T ? lane : 0);
+        // lanes = (trial tl, entry part): 32 / kWT parts scan interleaved
+        // entries, merged by shuffles
+        constexpr int NP = 32 / kWT;
+        const int tl = lane & (kWT - 1), part = lane / kWT;
+        const int j = tp0 + (tl < T ? tl : 0);
         const uint32_t A = sA[j], B = sB[j];
         uint32_t m[S];
 #pragma unroll
         for (int i = 0; i < S; ++i) m[i] = 0xFFFFFFFFu;
-        int e = 0;
-        for (; e + 4 <= ll; e += 4) {
-          const uint32_t x0 = src[e], x1 = src[e + 1], x2 = src[e + 2], x3 = src[e + 3];
+        int e = part;
+        for (; e + 3 * NP < ll; e += 4 * NP) {
+          const uint32_t x0 = src[e], x1 = src[e + NP], x2 = src[e + 2 * NP], x3 = src[e + 3 * NP];
           insert_min<S>(m, m31_hash(A, B, x0));
           insert_min<S>(m, m31_hash(A, B, x1));
           insert_min<S>(m, m31_hash(A, B, x2));
           insert_min<S>(m, m31_hash(A, B, x3));
         }
-        for (; e < ll; ++e) insert_min<S>(m, m31_hash(A, B, src[e]));
-        if (lane < T) sK[lane * kWin + lrow] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
+        for (; e < ll; e += NP) insert_min<S>(m, m31_hash(A, B, src[e]));
+        for (int o = kWT; o < 32; o <<= 1) {
+          uint32_t x[S];
+#pragma unroll
+          for (int i = 0; i < S; ++i) x[i] = __shfl_xor_sync(0xffffffffu, m[i], o);
+#pragma unroll
+          for (int i = 0; i < S; ++i) insert_min<S>(m, x[i]);
+        }
+        if (part == 0 && tl < T) sK[tl * kWin + lrow] = fmix(shingle_id<S>(m, a.seed, a.t0 + j));
       }
       __syncthreads();
       // natural-order write-out: trial j's kWin keys are contiguous
@@ -692,7 +702,7 @@ __global__ void __launch_bounds__(kWin, 3) minhash_win_kernel(const __grid_const
 
 template <int S>
 cudaError_t launch_win(MhParams &P, int num_sms, cudaStream_t st) {
-  const size_t smem = (size_t)32 * kWin * 8 + (size_t)2 * P.a.nt * 4;
+  const size_t smem = (size_t)kWT * kWin * 8 + (size_t)2 * P.a.nt * 4;
   auto kern = minhash_win_kernel<S>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -717,7 +727,10 @@ cudaError_t launch_win(MhParams &P, int num_sms, cudaStream_t st) {
 // Short rows (pass II) take 16-row tiles: a trial's keys of one tile are a
 // full 128 B line; long rows (pass I) keep 8-row tiles (the stage holds them).
 // SG_MH_WIN=1 (A/B): the windowed row-per-lane kernel instead of the 16-row
-// tile kernel for pass II (measured slower on gos2m: hash2 51.5 vs 43.2 ms).
+// tile kernel for pass II (parity-green, measured slower on gos2m: hash2 49.9
+// vs 43.9 ms; ncu: 11.1e9 vs 10.9e9 warp-instructions per 64-trial chunk —
+// the per-(row, trial) key mixing, staging and the long rows' lane = trial
+// scans cost as much as the tile kernel's row overheads).
 static bool use_tile16() {
   static const bool v = [] {
     const char *e = getenv("SG_MH_WIN");
