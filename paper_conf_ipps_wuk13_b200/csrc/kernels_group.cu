@@ -147,32 +147,23 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
   __syncthreads();
   {
     // bin-major, warp-minor exclusive prefix: thread t owns bin t (nb <= 256)
-    // (all loads of a column before its stores: no load-after-store chain)
     const int t = threadIdx.x;
     uint32_t run = 0;
     if (t < nb) {
-      uint32_t c[kSWarps];
-#pragma unroll
-      for (int x = 0; x < kSWarps; ++x) c[x] = S.cnt[x * nb + t];
-#pragma unroll
+#pragma unroll 4
       for (int x = 0; x < kSWarps; ++x) {
-        const uint32_t v = c[x];
-        c[x] = run;
-        run += v;
+        const uint32_t c = S.cnt[x * nb + t];
+        S.cnt[x * nb + t] = (uint16_t)run;
+        run += c;
       }
-#pragma unroll
-      for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + t] = (uint16_t)c[x];
     }
     int64_t all;
     const int64_t ex = block_excl_scan<int64_t>((int64_t)run, S.ws, &all);
     if (t < nb) {
       S.sbst[t] = (uint32_t)ex;
       S.off[t] = obase(t) - ex;
-      uint32_t c[kSWarps];
-#pragma unroll
-      for (int x = 0; x < kSWarps; ++x) c[x] = S.cnt[x * nb + t];
-#pragma unroll
-      for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + t] = (uint16_t)(c[x] + (uint32_t)ex);
+#pragma unroll 4
+      for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + t] += (uint16_t)ex;
     }
     if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
@@ -446,38 +437,6 @@ __global__ void binscan_kernel(const __grid_constant__ GroupArgs g) {
 }
 
 // ---- 3. stable coarse scatter (persistent) ------------------------------------
-// A chunk's table entries (loaded an iteration ahead of its keys, so the
-// keys' addresses are ready when they are needed).
-struct ChunkMeta {
-  int64_t i0 = 0, in0 = 0;
-  int len = 0, trial = 0;
-};
-
-__device__ __forceinline__ ChunkMeta chunk_meta(const GroupArgs &g, int64_t k) {
-  ChunkMeta m;
-  if (k < g.plan.nchunks) {
-    m.i0 = g.plan.chunk_i0[k];
-    m.in0 = g.plan.chunk_in0[k];
-    m.len = g.plan.chunk_len[k];
-    m.trial = g.plan.chunk_trial[k];
-  }
-  return m;
-}
-
-__device__ __forceinline__ void load_chunk(const GroupArgs &g, const ChunkMeta &m,
-                                           uint64_t (&kk)[kPerLane], uint32_t (&vv)[kPerLane]) {
-  const int64_t i0 = m.i0, in0 = m.in0;
-  const int len = m.len;
-#pragma unroll
-  for (int u = 0; u < kPerLane; ++u) {
-    const int e = elem_of(u);
-    if (e < len) {
-      kk[u] = g.keys[in0 + e];
-      vv[u] = val_at(g, in0 + e, i0 + e);
-    }
-  }
-}
-
 __device__ __forceinline__ void load_chunk(const GroupArgs &g, int64_t k, uint64_t (&kk)[kPerLane],
                                            uint32_t (&vv)[kPerLane]) {
   const int64_t i0 = g.plan.chunk_i0[k];
@@ -508,21 +467,17 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
   uint64_t kk[kPerLane];
   uint32_t vv[kPerLane];
   int64_t k = blockIdx.x;
-  ChunkMeta cur = chunk_meta(g, k);
-  if (k < g.plan.nchunks) load_chunk(g, cur, kk, vv);
-  ChunkMeta nxt = chunk_meta(g, k + gridDim.x);
+  if (k < g.plan.nchunks) load_chunk(g, k, kk, vv);
   while (k < g.plan.nchunks) {
-    const int j = cur.trial;
-    const int len = cur.len;
+    const int j = g.plan.chunk_trial[k];
+    const int len = g.plan.chunk_len[k];
     const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];   // scratch segment start
     int64_t gb = 0;
     if (threadIdx.x < nb)
       gb = sseg + (int64_t)g.bstart1[(int64_t)j * nb + threadIdx.x] + g.counts[k * nb + threadIdx.x];
     split_place<false, C8 ? kMaxFan : 0, AT>(S, len, nb, kk, vv, bin, [&](int) { return gb; });
     const int64_t kn = k + gridDim.x;
-    if (kn < g.plan.nchunks) load_chunk(g, nxt, kk, vv);   // in flight during the stores
-    cur = nxt;
-    nxt = chunk_meta(g, kn + gridDim.x);                   // the tables one chunk further
+    if (kn < g.plan.nchunks) load_chunk(g, kn, kk, vv);   // in flight during the stores
     if (!C8 && g.peer_keys) {
       // fused exchange: bin d = owner rank d, stored straight into its
       // receive buffers (NVLink / NVSwitch peer stores; same device for the
