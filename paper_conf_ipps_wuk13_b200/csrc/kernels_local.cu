@@ -401,8 +401,12 @@ static_assert(kCntPerThread == 8, "counter scan assumes 8 per thread");
 
 // One stable multi-split pass over n <= 4096 elements: warp w owns the
 // positions [w*seg, (w+1)*seg) of the current order src (identity if null)
-// and writes the new order to dst, stable on digit(key).
-template <typename DIG>
+// and writes the new order to dst, stable on digit(key).  ATOMIC: every
+// element counts and takes its slot with its own shared atomic on the
+// (digit, warp) counter instead of __match_any_sync peers (stable when the
+// hardware serves one instruction's conflicting lanes in lane order, as
+// measured; the caller's (key, member) verification repairs it otherwise).
+template <bool ATOMIC, typename DIG>
 __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *src, uint16_t *dst,
                                          DIG digit) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -410,6 +414,53 @@ __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *sr
   const int seg = (n + kLWarps - 1) / kLWarps;     // <= 512
   reinterpret_cast<uint4 *>(S.cnt)[threadIdx.x] = make_uint4(0, 0, 0, 0);
   __syncthreads();
+  if (ATOMIC) {
+    uint32_t *cw = reinterpret_cast<uint32_t *>(S.cnt);
+    const int seg_lo = w * seg, seg_hi = min(n, seg_lo + seg);
+    for (int pos = seg_lo + lane; pos < seg_hi; pos += 32) {
+      const int idx = (int)digit(S.K[src ? src[pos] : pos]) * kLWarps + w;
+      atomicAdd(cw + (idx >> 1), 1u << ((idx & 1) << 4));
+    }
+    __syncthreads();
+    {
+      uint4 *c4 = reinterpret_cast<uint4 *>(S.cnt);
+      uint4 v = c4[threadIdx.x];
+      uint16_t *c = reinterpret_cast<uint16_t *>(&v);
+      uint32_t s = 0, run[kCntPerThread];
+#pragma unroll
+      for (int x = 0; x < kCntPerThread; ++x) {
+        run[x] = s;
+        s += c[x];
+      }
+      int64_t tot;
+      const int64_t ex = block_excl_scan<int64_t>((int64_t)s, S.ws, &tot);
+#pragma unroll
+      for (int x = 0; x < kCntPerThread; ++x) c[x] = (uint16_t)(ex + run[x]);
+      c4[threadIdx.x] = v;
+    }
+    __syncthreads();
+    for (int pos0 = seg_lo; pos0 < seg_hi; pos0 += 4 * 32) {
+      uint32_t el[4], o[4];
+      int id[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int pos = pos0 + u * 32 + lane;
+        el[u] = 0;
+        o[u] = 0;
+        id[u] = 0;
+        if (pos < seg_hi) {
+          el[u] = src ? src[pos] : (uint32_t)pos;
+          id[u] = (int)digit(S.K[el[u]]) * kLWarps + w;
+          o[u] = atomicAdd(cw + (id[u] >> 1), 1u << ((id[u] & 1) << 4));
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (pos0 + u * 32 + lane < seg_hi) dst[(o[u] >> ((id[u] & 1) << 4)) & 0xFFFFu] = (uint16_t)el[u];
+    }
+    __syncthreads();
+    return;
+  }
   uint32_t *pr = S.peers + w * kPerLane * 32;     // match masks of this warp
   const int seg_lo = w * seg, seg_hi = min(n, seg_lo + seg);
   for (int pos = seg_lo + lane; pos - lane < seg_hi; pos += 32) {   // warp-uniform trip count
@@ -461,6 +512,7 @@ __device__ __forceinline__ void lsd_pass(LocalSmem &S, int n, const uint16_t *sr
   __syncthreads();
 }
 
+template <bool ATOMIC>
 __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   LocalSmem &S = *reinterpret_cast<LocalSmem *>(smraw);
@@ -479,13 +531,15 @@ __global__ void __launch_bounds__(kLThreads, 2) local_kernel(const __grid_consta
     }
     cp_async_wait_all();
     // (lsd_pass begins with a barrier after zeroing its counters)
-    lsd_pass(S, n, nullptr, S.perm[0],
-             [&](uint64_t key) { return (uint32_t)((key << (bits + 8)) >> 56); });
-    lsd_pass(S, n, S.perm[0], S.perm[1],
-             [&](uint64_t key) { return (uint32_t)((key << bits) >> 56); });
+    lsd_pass<ATOMIC>(S, n, nullptr, S.perm[0],
+                     [&](uint64_t key) { return (uint32_t)((key << (bits + 8)) >> 56); });
+    lsd_pass<ATOMIC>(S, n, S.perm[0], S.perm[1],
+                     [&](uint64_t key) { return (uint32_t)((key << bits) >> 56); });
     const uint16_t *pm = S.perm[1];
     const uint64_t *K = S.K;
-    auto d16 = [&](uint64_t key) { return (uint32_t)((key << bits) >> 48); };
+    // repair runs: equal 16 sorted bits, or (ATOMIC: the last pass may be
+    // unstable only inside one high digit) equal high digit
+    auto d16 = [&](uint64_t key) { return (uint32_t)((key << bits) >> (ATOMIC ? 56 : 48)); };
     // ---- rare: distinct keys sharing the 16 bits out of key order -> a
     // stable insertion sort of that run (registered once via its start bit)
     for (int i = threadIdx.x; i < (kLocalCap / 32 + 2); i += blockDim.x) S.hb[i] = 0;
@@ -644,11 +698,17 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   }
   // CTA tier over the mid list (length read on the device)
   {
+    // SG_LOCAL_CTA_ATOMIC=0 (A/B): the match-based placements
+    static const bool cat = [] {
+      const char *e = getenv("SG_LOCAL_CTA_ATOMIC");
+      return !(e && atoi(e) == 0);
+    }();
     const size_t smem = sizeof(LocalSmem);
-    cudaError_t e = cudaFuncSetAttribute(local_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem);
+    const void *fn = cat ? (const void *)local_kernel<true> : (const void *)local_kernel<false>;
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    local_kernel<<<num_sms * 2, kLThreads, smem, st>>>(g);
+    if (cat) local_kernel<true><<<num_sms * 2, kLThreads, smem, st>>>(g);
+    else local_kernel<false><<<num_sms * 2, kLThreads, smem, st>>>(g);
     ++g_launches;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }

@@ -288,6 +288,20 @@ def test_many_bins_and_tiny_buckets(B, target, v3, monkeypatch):
     assert_parity(out, ref, report=False)
 
 
+@pytest.mark.parametrize("target", ["2048", "3500"])
+def test_cta_tier_buckets(B, target, monkeypatch):
+    """Buckets of 1,025-4,096 pairs (the CTA tier, which sorts every level-II
+    bucket of the 640M-edge config): atomic LSD placements, then the full
+    (key, member) verification and repair, element by element against the
+    oracle."""
+    g = SG.make("small")
+    cfg = SG.CONFIGS["small"]
+    monkeypatch.setenv("SG_GROUP_TARGET", target)
+    out, ref = run_both(B, g, cfg["s1"], cfg["c1"], cfg["seed1"], cfg["s2"], cfg["c2"], cfg["seed2"],
+                        report=False)
+    assert_parity(out, ref, report=False)
+
+
 def test_invalid_csr_rejected(B):
     g = SG.random_graph(200, 900, seed=2)
     r = int(np.argmax(np.diff(g.row_ptr) >= 2))
