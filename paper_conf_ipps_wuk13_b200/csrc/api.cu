@@ -106,9 +106,12 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
     return;
   }
   void *p = nullptr;
+  const auto t0 = std::chrono::steady_clock::now();
+  ++g->n_pool_allocs;
   cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
+    ++g->n_cache_releases;
     cache_release(g);
     e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   }
@@ -117,10 +120,12 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
     // (e.g. after a step with another (s, c)): return them to the device and
     // map the request afresh (the handle's private pool only)
     cudaGetLastError();
+    ++g->n_trims;
     cudaStreamSynchronize(g->stream);
     cudaMemPoolTrimTo(g->pool, 0);
     e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   }
+  g->alloc_host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   if (e != cudaSuccess) {
     cudaGetLastError();
     size_t fr = 0, tot = 0;
@@ -479,14 +484,14 @@ struct GroupScratch {
   DBuf p_trial, p_in0, p_len, p_row0, p_chunk0, seg, trial_chunk0;
   DBuf chunk_i0, chunk_in0, chunk_len, chunk_trial;
   DBuf counts, bstart1, bsize1, bstart, bsize, akeys, avals, bkeys, bvals, big_list, big_count;
-  DBuf seg_pos, seg_len;
+  DBuf seg_pos, seg_len, fbin;
 };
 
 void free_scratch(sg_graph *g, GroupScratch &S) {
   for (DBuf *b : {&S.p_trial, &S.p_in0, &S.p_len, &S.p_row0, &S.p_chunk0, &S.seg, &S.trial_chunk0,
                   &S.chunk_i0, &S.chunk_in0, &S.chunk_len, &S.chunk_trial,
                   &S.counts, &S.bstart1, &S.bsize1, &S.bstart, &S.bsize, &S.akeys, &S.avals,
-                  &S.bkeys, &S.bvals, &S.big_list, &S.big_count, &S.seg_pos, &S.seg_len})
+                  &S.bkeys, &S.bvals, &S.big_list, &S.big_count, &S.seg_pos, &S.seg_len, &S.fbin})
     dfree(g, *b);
 }
 
@@ -497,7 +502,7 @@ double scratch_per_pair(int64_t maxseg) {
   if (!use_group_v1()) return 13.9;          // v3: one partitioned copy (8 B key + 4 B value) + segment list
   int32_t b, b1;
   group_bits(maxseg, &b, &b1);
-  return b == b1 ? 12.5 : 24.5;
+  return b == b1 ? 12.5 : (b == 16 && b1 == 8 ? 25.5 : 24.5);   // + the fine-digit bytes
 }
 
 // A contiguous run of pre-group pairs of one (local) trial: keys / explicit
@@ -597,11 +602,14 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   need(S.bsize1, (size_t)(nt * nb1) * 4);
   need(S.akeys, (size_t)npairs * 8);
   need(S.avals, (size_t)npairs * 4);
+  // fine digits as bytes for the fine split's histogram (16-bit plans)
+  const bool fb = two && bits == 16 && bits1 == 8 && !getenv("SG_NO_FBIN");
   if (two) {
     need(S.bstart, (size_t)(nt * nbins) * 4);
     need(S.bsize, (size_t)(nt * nbins) * 4);
     need(S.bkeys, (size_t)npairs * 8);
     need(S.bvals, (size_t)npairs * 4);
+    if (fb) need(S.fbin, (size_t)npairs);
   }
   need(S.big_list, (size_t)(nt * nbins) * 8);             // big + mid lists
   need(S.big_count, 8);                                    // big + mid counts
@@ -627,6 +635,7 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   a.bsize = two ? ptr<uint32_t>(S.bsize) : a.bsize1;
   a.bkeys = two ? ptr<uint64_t>(S.bkeys) : a.akeys;
   a.bvals = two ? ptr<uint32_t>(S.bvals) : a.avals;
+  a.fbin = fb ? ptr<uint8_t>(S.fbin) : nullptr;
   a.big_list = ptr<uint32_t>(S.big_list);
   a.big_count = ptr<uint32_t>(S.big_count);
   a.mid_list = a.big_list + nt * nbins;
@@ -1543,6 +1552,14 @@ sg_status group_by_shingle(sg_graph *g) {
 
 sg_status shingle_graph_reset(sg_graph *g) {
   return guarded(g, [&] {
+    static const bool log = getenv("SG_ALLOC_LOG") != nullptr;
+    if (log)
+      fprintf(stderr, "sg alloc: pool allocations %lld, cache releases %lld, pool trims %lld, "
+                      "host ms in pool calls %.2f, live %.2f GB, cached %.2f GB in %zu blocks\n",
+              (long long)g->n_pool_allocs, (long long)g->n_cache_releases, (long long)g->n_trims,
+              g->alloc_host_ms, g->bytes_live / 1e9, g->bytes_cached / 1e9, g->cache.size());
+    g->n_pool_allocs = g->n_cache_releases = g->n_trims = 0;
+    g->alloc_host_ms = 0;
     for (int l = 0; l < 2; ++l) {
       free_pass(g, g->pass[l]);
       free_groups(g, g->grp[l]);

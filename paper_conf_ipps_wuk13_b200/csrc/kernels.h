@@ -105,6 +105,8 @@ struct GroupArgs {
   uint32_t *bsize;             // [c][nbins]
   uint64_t *akeys;             // [npairs] coarse-bucketed pairs
   uint32_t *avals;
+  uint8_t *fbin = nullptr;     // [npairs] fine digit (key bits 48..55) of the coarse-bucketed
+                               // pairs, 16-bit two-level plans only (or nullptr)
   // fused exchange (SG_DIST_PEER): owner partition writes bin d's pairs into
   // rank d's receive buffers (device arrays of nb1 peer pointers) instead of
   // akeys / avals

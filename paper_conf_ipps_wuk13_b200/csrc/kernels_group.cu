@@ -248,12 +248,14 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
 template <typename BIN>
 __device__ __forceinline__ void emit_runs(const SplitSmem &S, int len, BIN bin_of,
                                           uint64_t *__restrict__ outK,
-                                          uint32_t *__restrict__ outV) {
+                                          uint32_t *__restrict__ outV,
+                                          uint8_t *__restrict__ outF = nullptr) {
   for (int p = threadIdx.x; p < len; p += kSThreads) {
     const uint64_t key = S.K[p];
     const int64_t o = S.off[bin_of(key)] + p;
     outK[o] = key;
     outV[o] = S.V[p];
+    if (outF) outF[o] = (uint8_t)(key >> 48);   // the fine digit of 16-bit plans
   }
 }
 
@@ -490,7 +492,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
         g.peer_vals[d][o] = S.V[p];
       }
     } else {
-      emit_runs(S, len, bin, g.akeys, g.avals);
+      emit_runs(S, len, bin, g.akeys, g.avals, C8 ? g.fbin : nullptr);
     }
     __syncthreads();
     k = kn;
@@ -523,7 +525,32 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   // fine-bucket totals (order-free), starts, sizes
   for (int i = threadIdx.x; i < nb2; i += blockDim.x) S.tot[i] = 0;
   __syncthreads();
-  {
+  if (F8 && g.fbin) {
+    // the coarse scatter wrote each pair's fine digit as one byte: count
+    // 1 B per pair instead of re-reading the 8-B keys (aligned words, two
+    // in flight per thread; the unaligned head and tail byte by byte)
+    const uint8_t *__restrict__ fb = g.fbin + sseg + st1;
+    const int head = (int)((4 - ((uintptr_t)fb & 3)) & 3);
+    const int h = (int)min((int64_t)head, n);
+    if ((int)threadIdx.x < h) atomicAdd(&S.tot[fb[threadIdx.x]], 1u);
+    const uint32_t *__restrict__ fw = reinterpret_cast<const uint32_t *>(fb + h);
+    const int64_t nw = (n - h) >> 2;
+    int64_t i = threadIdx.x;
+    for (; i + kSThreads < nw; i += 2 * kSThreads) {
+      const uint32_t w0 = fw[i], w1 = fw[i + kSThreads];
+#pragma unroll
+      for (int x = 0; x < 4; ++x) atomicAdd(&S.tot[(w0 >> (8 * x)) & 0xFFu], 1u);
+#pragma unroll
+      for (int x = 0; x < 4; ++x) atomicAdd(&S.tot[(w1 >> (8 * x)) & 0xFFu], 1u);
+    }
+    for (; i < nw; i += kSThreads) {
+      const uint32_t w0 = fw[i];
+#pragma unroll
+      for (int x = 0; x < 4; ++x) atomicAdd(&S.tot[(w0 >> (8 * x)) & 0xFFu], 1u);
+    }
+    const int64_t t0 = h + 4 * nw;
+    if ((int64_t)threadIdx.x < n - t0) atomicAdd(&S.tot[fb[t0 + threadIdx.x]], 1u);
+  } else {
     // four loads in flight per thread
     int64_t i = threadIdx.x;
     for (; i + 3 * kSThreads < n; i += 4 * kSThreads) {

@@ -698,10 +698,12 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   }
   // CTA tier over the mid list (length read on the device)
   {
-    // SG_LOCAL_CTA_ATOMIC=0 (A/B): the match-based placements
+    // SG_LOCAL_CTA_ATOMIC=1 (A/B): atomic placements (parity-green; measured
+    // slower on the 640M-edge config, whose level-II buckets all take this
+    // tier: local2 533.6 vs 521.1 ms)
     static const bool cat = [] {
       const char *e = getenv("SG_LOCAL_CTA_ATOMIC");
-      return !(e && atoi(e) == 0);
+      return e && atoi(e) != 0;
     }();
     const size_t smem = sizeof(LocalSmem);
     const void *fn = cat ? (const void *)local_kernel<true> : (const void *)local_kernel<false>;

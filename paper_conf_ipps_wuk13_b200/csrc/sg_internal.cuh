@@ -196,4 +196,7 @@ struct sg_graph {
   } plan_memo[2];
   std::vector<sg::DBuf> cache;  // freed blocks kept for reuse (best fit)
   int64_t bytes_cached = 0;
+  // allocation diagnostics since the last reset (SG_ALLOC_LOG prints them)
+  int64_t n_pool_allocs = 0, n_cache_releases = 0, n_trims = 0;
+  double alloc_host_ms = 0;
 };
