@@ -502,7 +502,7 @@ double scratch_per_pair(int64_t maxseg) {
   if (!use_group_v1()) return 13.9;          // v3: one partitioned copy (8 B key + 4 B value) + segment list
   int32_t b, b1;
   group_bits(maxseg, &b, &b1);
-  return b == b1 ? 12.5 : (b == 16 && b1 == 8 ? 25.5 : 24.5);   // + the fine-digit bytes
+  return b == b1 ? 12.5 : (b == 16 && b1 == 8 && getenv("SG_FBIN") ? 25.5 : 24.5);   // + fine bytes
 }
 
 // A contiguous run of pre-group pairs of one (local) trial: keys / explicit
@@ -603,7 +603,9 @@ void group_pieces(sg_graph *g, const uint64_t *keys, const std::vector<Piece> &p
   need(S.akeys, (size_t)npairs * 8);
   need(S.avals, (size_t)npairs * 4);
   // fine digits as bytes for the fine split's histogram (16-bit plans)
-  const bool fb = two && bits == 16 && bits1 == 8 && !getenv("SG_NO_FBIN");
+  // (opt-in SG_FBIN=1: measured on gos2m fine 67.3 -> 62.9 ms but the
+  // coarse scatter's byte stores 76.7 -> 82.5 ms)
+  const bool fb = two && bits == 16 && bits1 == 8 && getenv("SG_FBIN");
   if (two) {
     need(S.bstart, (size_t)(nt * nbins) * 4);
     need(S.bsize, (size_t)(nt * nbins) * 4);

@@ -40,8 +40,8 @@ constexpr int kPerLane = kChunk / kSThreads;   // 8
 constexpr int kSeg = kChunk / kSWarps;         // 256 consecutive elements per warp
 constexpr int kMaxFan = 256;                   // bins of one split pass
 constexpr int kCoarseBits = 8;
-constexpr int kMaxBits = 16;                   // final buckets per trial <= 65536
-constexpr int kMaxFine = 1 << (kMaxBits - kCoarseBits);
+constexpr int kMaxBits = 18;                   // final buckets per trial <= 2^18
+constexpr int kMaxFine = 1 << (kMaxBits - kCoarseBits);   // fan-out of the fine split (1024)
 
 // Coarse bin = floor(key * nb / 2^64): the top log2(nb) key bits when nb is a
 // power of two (buckets), contiguous key ranges for any nb (owner ranks).
@@ -81,9 +81,9 @@ __device__ __forceinline__ int elem_of(int u) {
 struct SplitSmem {
   uint64_t K[kChunk];                  // chunk, bucket-major after the split
   uint32_t V[kChunk];
-  uint16_t cnt[kSWarps * kMaxFan];     // [warp][bin] running positions
-  uint32_t sbst[kMaxFan + 1];          // bin starts within the chunk
-  int64_t off[kMaxFan];                // output position - chunk position, per bin
+  uint16_t cnt[kSWarps * kMaxFine];    // [warp][bin] running positions
+  uint32_t sbst[kMaxFine + 1];         // bin starts within the chunk
+  int64_t off[kMaxFine];               // output position - chunk position, per bin
   int64_t gcur[kMaxFine];              // scatter2: running fine-bucket cursors
   uint32_t tot[kMaxFine];              // scatter2: fine-bucket totals
   int64_t ws[33];
@@ -146,24 +146,40 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
   }
   __syncthreads();
   {
-    // bin-major, warp-minor exclusive prefix: thread t owns bin t (nb <= 256)
+    // bin-major, warp-minor exclusive prefix: thread t owns bins
+    // [t*BPT, (t+1)*BPT) (BPT = 1 up to 512 bins, 2 for the 1024-bin fine split)
+    constexpr int BPTC = NBC > kSThreads ? (NBC + kSThreads - 1) / kSThreads : 1;
+    const int BPT = NBC > 0 ? BPTC : (nb + kSThreads - 1) / kSThreads;
     const int t = threadIdx.x;
-    uint32_t run = 0;
-    if (t < nb) {
+    uint32_t tsum = 0, bt[2] = {0, 0};
+#pragma unroll
+    for (int i = 0; i < 2; ++i) {
+      const int b = t * BPT + i;
+      if (i < BPT && b < nb) {
+        uint32_t run = 0;
 #pragma unroll 4
-      for (int x = 0; x < kSWarps; ++x) {
-        const uint32_t c = S.cnt[x * nb + t];
-        S.cnt[x * nb + t] = (uint16_t)run;
-        run += c;
+        for (int x = 0; x < kSWarps; ++x) {
+          const uint32_t c = S.cnt[x * nb + b];
+          S.cnt[x * nb + b] = (uint16_t)run;
+          run += c;
+        }
+        bt[i] = run;
+        tsum += run;
       }
     }
     int64_t all;
-    const int64_t ex = block_excl_scan<int64_t>((int64_t)run, S.ws, &all);
-    if (t < nb) {
-      S.sbst[t] = (uint32_t)ex;
-      S.off[t] = obase(t) - ex;
+    const int64_t ex = block_excl_scan<int64_t>((int64_t)tsum, S.ws, &all);
+    int64_t acc = ex;
+#pragma unroll
+    for (int i = 0; i < 2; ++i) {
+      const int b = t * BPT + i;
+      if (i < BPT && b < nb) {
+        S.sbst[b] = (uint32_t)acc;
+        S.off[b] = obase(b) - acc;
 #pragma unroll 4
-      for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + t] += (uint16_t)ex;
+        for (int x = 0; x < kSWarps; ++x) S.cnt[x * nb + b] += (uint16_t)acc;
+        acc += bt[i];
+      }
     }
     if (t == 0) S.sbst[nb] = (uint32_t)len;
   }
@@ -500,9 +516,11 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
 }
 
 // ---- 4. stable second-level scatter (one CTA per coarse bucket) ----------------
-// F8: bits == 16 with an 8-bit coarse level (the level-II plans of the 2M and
+// FB > 0: a plan with an 8-bit coarse level and FB fine bits known at compile
+// time (FB = 8: bits == 16, the level-II plans of the 2M and 640M configs;
+// FB = 7: bits == 15, hub2m):
 // 640M configs): fine digit = key bits 48..55 by a constant shift.
-template <bool F8, int AT>
+template <int FB, int AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
   SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
@@ -510,7 +528,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   const int64_t nb1 = g.plan.nb1;
   const int j = (int)(q1 / nb1);
   const int b1 = (int)(q1 % nb1);
-  const int bits = F8 ? 16 : g.plan.bits, bits2 = F8 ? 8 : g.plan.bits - g.plan.bits1;
+  const int bits = FB ? 8 + FB : g.plan.bits, bits2 = FB ? FB : g.plan.bits - g.plan.bits1;
   const int nb2 = 1 << bits2;
   const uint32_t mask2 = (uint32_t)nb2 - 1u;
   const int64_t sseg = g.plan.seg[j] - g.plan.seg[0];
@@ -519,13 +537,13 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   const uint64_t *__restrict__ K = g.akeys + sseg + st1;
   const uint32_t *__restrict__ V = g.avals + sseg + st1;
   auto fine = [&](uint64_t key) {
-    if (F8) return (uint32_t)(key >> 48) & 0xFFu;
+    if (FB) return (uint32_t)(key >> (56 - FB)) & ((1u << FB) - 1u);
     return top_bits(key, bits) & mask2;
   };
   // fine-bucket totals (order-free), starts, sizes
   for (int i = threadIdx.x; i < nb2; i += blockDim.x) S.tot[i] = 0;
   __syncthreads();
-  if (F8 && g.fbin) {
+  if (FB == 8 && g.fbin) {
     // the coarse scatter wrote each pair's fine digit as one byte: count
     // 1 B per pair instead of re-reading the 8-B keys (aligned words, two
     // in flight per thread; the unaligned head and tail byte by byte)
@@ -564,15 +582,23 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   }
   __syncthreads();
   {
-    const int d = threadIdx.x;
-    const int64_t v = d < nb2 ? S.tot[d] : 0;
+    // thread t owns fine bins [t*BPT, (t+1)*BPT)
+    const int BPT = (nb2 + kSThreads - 1) / kSThreads;
+    const int t = threadIdx.x;
+    int64_t v[2] = {0, 0};
+    for (int i = 0; i < BPT; ++i)
+      if (t * BPT + i < nb2) v[i] = S.tot[t * BPT + i];
     int64_t all;
-    const int64_t ex = block_excl_scan<int64_t>(v, S.ws, &all);
-    if (d < nb2) {
-      const int64_t qf = (int64_t)j * g.plan.nbins + ((int64_t)b1 << bits2) + d;
-      g.bstart[qf] = st1 + (uint32_t)ex;
-      g.bsize[qf] = (uint32_t)v;
-      S.gcur[d] = sseg + st1 + ex;
+    int64_t ex = block_excl_scan<int64_t>(v[0] + v[1], S.ws, &all);
+    for (int i = 0; i < BPT; ++i) {
+      const int d = t * BPT + i;
+      if (d < nb2) {
+        const int64_t qf = (int64_t)j * g.plan.nbins + ((int64_t)b1 << bits2) + d;
+        g.bstart[qf] = st1 + (uint32_t)ex;
+        g.bsize[qf] = (uint32_t)v[i];
+        S.gcur[d] = sseg + st1 + ex;
+      }
+      ex += v[i];
     }
   }
   __syncthreads();
@@ -592,7 +618,7 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_con
   if (n > 0) load(0);
   for (int64_t c0 = 0; c0 < n; c0 += kChunk) {
     const int len = (int)min((int64_t)kChunk, n - c0);
-    split_place<true, F8 ? kMaxFan : 0, AT>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
+    split_place<true, FB ? (1 << FB) : 0, AT>(S, len, nb2, kk, vv, fine, [&](int d) { return S.gcur[d]; });
     if (c0 + kChunk < n) load(c0 + kChunk);
     emit_runs(S, len, fine, g.bkeys, g.bvals);
     // advance the fine cursors by this sub-chunk's counts
@@ -768,13 +794,17 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
   const int64_t nq1 = (int64_t)g.plan.c * g.plan.nb1;
   if (nq1 == 0 || g.plan.bits == g.plan.bits1) return cudaSuccess;
   if (g.plan.bits - g.plan.bits1 > kMaxBits - kCoarseBits) return cudaErrorInvalidValue;
-  const bool f8 = g.plan.bits == 16 && g.plan.bits1 == kCoarseBits;
+  const int fbits = (g.plan.bits1 == kCoarseBits &&
+                     (g.plan.bits == 18 || g.plan.bits == 16 || g.plan.bits == 15))
+                        ? g.plan.bits - kCoarseBits : 0;
   const int mode = split_mode(true);
   const void *fn = nullptr;
-  switch ((f8 ? 4 : 0) + mode) {
-#define SG_SC(C, M) case (C ? 4 : 0) + M: fn = (const void *)scatter2_kernel<C, M>; break;
-    SG_SC(true, 0) SG_SC(true, 1) SG_SC(true, 2) SG_SC(true, 3)
-    SG_SC(false, 0) SG_SC(false, 1) SG_SC(false, 2) SG_SC(false, 3)
+  switch (fbits * 4 + mode) {
+#define SG_SC(F, M) case F * 4 + M: fn = (const void *)scatter2_kernel<F, M>; break;
+    SG_SC(10, 0) SG_SC(10, 1) SG_SC(10, 2) SG_SC(10, 3)
+    SG_SC(8, 0) SG_SC(8, 1) SG_SC(8, 2) SG_SC(8, 3)
+    SG_SC(7, 0) SG_SC(7, 1) SG_SC(7, 2) SG_SC(7, 3)
+    SG_SC(0, 0) SG_SC(0, 1) SG_SC(0, 2) SG_SC(0, 3)
 #undef SG_SC
   }
   int per_sm = 1;

@@ -670,7 +670,7 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
   // warp tier over all buckets
   {
     const size_t smem = sizeof(WarpSmem) * kWWarps;
-    const bool b16 = g.plan.bits == 16;
+    const int bk = (g.plan.bits == 18 || g.plan.bits == 16 || g.plan.bits == 15) ? g.plan.bits : 0;
     // default: atomic placements + full-order verification (SG_LOCAL_ATOMIC=0:
     // the match-based stable placements, key-only tie check)
     // (forced on when the splits rank atomically: only the verifying tier
@@ -679,8 +679,13 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
       const char *e = getenv("SG_LOCAL_ATOMIC");
       return !(e && atoi(e) == 0) || split_atomic() > 0;
     }();
-    const void *fn = b16 ? (atom ? (const void *)warp_local_kernel<16, true> : (const void *)warp_local_kernel<16, false>)
-                         : (atom ? (const void *)warp_local_kernel<0, true> : (const void *)warp_local_kernel<0, false>);
+    const void *fn = nullptr;
+    switch (bk * 2 + (atom ? 1 : 0)) {
+#define SG_WL(B, A) case B * 2 + A: fn = (const void *)warp_local_kernel<B, A>; break;
+      SG_WL(18, 1) SG_WL(18, 0) SG_WL(16, 1) SG_WL(16, 0) SG_WL(15, 1) SG_WL(15, 0)
+      SG_WL(0, 1) SG_WL(0, 0)
+#undef SG_WL
+    }
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
@@ -689,10 +694,8 @@ cudaError_t group_local(const GroupArgs &g, int num_sms, cudaStream_t st) {
     per_sm = std::max(per_sm, 1);
     const int64_t want = (nq + kWWarps - 1) / kWWarps;
     const int grid = (int)std::min<int64_t>((int64_t)num_sms * per_sm, want);
-    if (b16 && atom) warp_local_kernel<16, true><<<grid, kWWarps * 32, smem, st>>>(g);
-    else if (b16) warp_local_kernel<16, false><<<grid, kWWarps * 32, smem, st>>>(g);
-    else if (atom) warp_local_kernel<0, true><<<grid, kWWarps * 32, smem, st>>>(g);
-    else warp_local_kernel<0, false><<<grid, kWWarps * 32, smem, st>>>(g);
+    void *args[] = {(void *)&g};
+    if ((e = cudaLaunchKernel(fn, dim3(grid), dim3(kWWarps * 32), args, smem, st)) != cudaSuccess) return e;
     ++g_launches;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }

@@ -271,7 +271,7 @@ def test_trial_chunking_under_memory_budget(B, budget_mb, monkeypatch):
 
 
 @pytest.mark.parametrize("v3", [False, True])
-@pytest.mark.parametrize("target", ["4", "40", "300"])
+@pytest.mark.parametrize("target", ["1", "4", "40", "300"])
 def test_many_bins_and_tiny_buckets(B, target, v3, monkeypatch):
     """SG_GROUP_TARGET shrinks the target bucket size so that the small graph
     takes the two-level partition (coarse scatter + per-bucket scatter) used

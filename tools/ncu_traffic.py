@@ -13,7 +13,7 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-GROUP_KERNELS = ("hist_kernel", "colscan_kernel", "binscan_kernel", "scatter_kernel", "scatter2_kernel",
+GROUP_KERNELS = ("hist_kernel", "hist_bytes_kernel", "colscan_kernel", "binscan_kernel", "scatter_kernel", "scatter2_kernel",
                  "warp_local_kernel", "local_kernel", "big_kernel")
 
 
