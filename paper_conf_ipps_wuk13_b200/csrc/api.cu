@@ -61,8 +61,18 @@ bool no_cache() {
   return v;
 }
 
+// Blocks above SG_CACHE_MAX_BYTES (default: no limit) go straight back to
+// the stream-ordered pool instead of the handle's best-fit cache.
+size_t cache_max_bytes() {
+  static const size_t v = [] {
+    const char *e = getenv("SG_CACHE_MAX_BYTES");
+    return e ? (size_t)atoll(e) : (size_t)-1;
+  }();
+  return v;
+}
+
 void cache_put(sg_graph *g, void *p, size_t bytes) {
-  if (no_cache()) {
+  if (no_cache() || bytes > cache_max_bytes()) {
     cudaFreeAsync(p, g->stream);
     return;
   }

@@ -78,16 +78,22 @@ __device__ __forceinline__ int elem_of(int u) {
   return (threadIdx.x >> 5) * kSeg + u * 32 + (threadIdx.x & 31);
 }
 
-struct SplitSmem {
+// MB: the largest fan-out the kernel uses (256 for the coarse scatter and
+// the <= 8-bit fine splits; 1024 for the 10-bit fine split of 18-bit plans:
+// 104 KB instead of 64 KB, which also shrinks L1 — measured: sizing every
+// split for 1024 bins slowed the gos2m fine split 66 -> 83 ms).
+template <int MB>
+struct SplitSmemT {
   uint64_t K[kChunk];                  // chunk, bucket-major after the split
   uint32_t V[kChunk];
-  uint16_t cnt[kSWarps * kMaxFine];    // [warp][bin] running positions
-  uint32_t sbst[kMaxFine + 1];         // bin starts within the chunk
-  int64_t off[kMaxFine];               // output position - chunk position, per bin
-  int64_t gcur[kMaxFine];              // scatter2: running fine-bucket cursors
-  uint32_t tot[kMaxFine];              // scatter2: fine-bucket totals
+  uint16_t cnt[kSWarps * MB];          // [warp][bin] running positions
+  uint32_t sbst[MB + 1];               // bin starts within the chunk
+  int64_t off[MB];                     // output position - chunk position, per bin
+  int64_t gcur[MB];                    // scatter2: running fine-bucket cursors
+  uint32_t tot[MB];                    // scatter2: fine-bucket totals
   int64_t ws[33];
 };
+using SplitSmem = SplitSmemT<kMaxFan>;
 
 // Rank the len <= kChunk pairs (kk, vv) of one chunk stably by bin_of(key) in
 // [0, nb) and place them bucket-major in S.K / S.V.  obase(b) gives the output
@@ -109,8 +115,8 @@ struct SplitSmem {
 //     peer masks as in 0 (stable);
 //  3: counts as in 2, placement by peer masks with the lowest peer taking
 //     the run's base by a returning atomic (no __syncwarp chain; stable).
-template <bool BALLOT, int NBC, int AT, typename BIN, typename OBASE>
-__device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
+template <bool BALLOT, int NBC, int AT, typename SM, typename BIN, typename OBASE>
+__device__ __forceinline__ void split_place(SM &S, int len, int nb_rt,
                                             const uint64_t (&kk)[kPerLane],
                                             const uint32_t (&vv)[kPerLane], BIN bin_of,
                                             OBASE obase) {
@@ -261,8 +267,8 @@ __device__ __forceinline__ void split_place(SplitSmem &S, int len, int nb_rt,
 
 // Write the placed chunk: consecutive threads take consecutive chunk
 // positions, which inside one bin are consecutive output positions.
-template <typename BIN>
-__device__ __forceinline__ void emit_runs(const SplitSmem &S, int len, BIN bin_of,
+template <typename SM, typename BIN>
+__device__ __forceinline__ void emit_runs(const SM &S, int len, BIN bin_of,
                                           uint64_t *__restrict__ outK,
                                           uint32_t *__restrict__ outV,
                                           uint8_t *__restrict__ outF = nullptr) {
@@ -523,7 +529,8 @@ __global__ void __launch_bounds__(kSThreads, 2) scatter_kernel(const __grid_cons
 template <int FB, int AT>
 __global__ void __launch_bounds__(kSThreads, 2) scatter2_kernel(const __grid_constant__ GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smraw[];
-  SplitSmem &S = *reinterpret_cast<SplitSmem *>(smraw);
+  using SM = SplitSmemT<(FB == 0 || FB > 8) ? kMaxFine : kMaxFan>;
+  SM &S = *reinterpret_cast<SM *>(smraw);
   const int64_t q1 = blockIdx.x;                 // (trial, coarse bucket)
   const int64_t nb1 = g.plan.nb1;
   const int j = (int)(q1 / nb1);
@@ -758,8 +765,7 @@ cudaError_t group_offsets(const GroupArgs &g, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-static cudaError_t split_attr(const void *fn, int *per_sm) {
-  const size_t smem = sizeof(SplitSmem);
+static cudaError_t split_attr(const void *fn, int *per_sm, size_t smem = sizeof(SplitSmem)) {
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, fn, kSThreads, smem);
@@ -807,11 +813,12 @@ cudaError_t group_scatter2(const GroupArgs &g, cudaStream_t st) {
     SG_SC(0, 0) SG_SC(0, 1) SG_SC(0, 2) SG_SC(0, 3)
 #undef SG_SC
   }
+  const size_t sm2 = (fbits == 0 || fbits > 8) ? sizeof(SplitSmemT<kMaxFine>) : sizeof(SplitSmem);
   int per_sm = 1;
-  cudaError_t e = split_attr(fn, &per_sm);
+  cudaError_t e = split_attr(fn, &per_sm, sm2);
   if (e != cudaSuccess) return e;
   void *args[] = {(void *)&g};
-  e = cudaLaunchKernel(fn, dim3((unsigned)nq1), dim3(kSThreads), args, sizeof(SplitSmem), st);
+  e = cudaLaunchKernel(fn, dim3((unsigned)nq1), dim3(kSThreads), args, sm2, st);
   if (e != cudaSuccess) return e;
   ++g_launches;
   return cudaGetLastError();
