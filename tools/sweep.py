@@ -48,10 +48,14 @@ def main():
     g = SG.make(args.config)
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
-    h = B.shingle_graph_create(g.row_ptr, g.col, dist={"rank": 0, "world": 1, "device": 0,
-                                                       "stream": stream.cuda_stream})
     for s in (int(x) for x in args.s.split(",")):
         for c in (int(x) for x in args.c.split(",")):
+            # a fresh handle (and memory pool) per point: the cached blocks of
+            # another (s, c) plan would otherwise turn the next point's first
+            # steps into pool releases and re-maps
+            h = B.shingle_graph_create(g.row_ptr, g.col, dist={"rank": 0, "world": 1, "device": 0,
+                                                               "stream": stream.cuda_stream})
+
             def step():
                 B.shingle_graph_reset(h)
                 B.shingle_pass(h, s, c, cfg["seed1"])
@@ -99,7 +103,7 @@ def main():
             except B.SGError as e:
                 line["error"] = str(e)
             print(json.dumps(line), flush=True)
-    B.shingle_graph_destroy(h)
+            B.shingle_graph_destroy(h)
 
 
 if __name__ == "__main__":
