@@ -349,9 +349,19 @@ void plan_pass(sg_graph *g, PassOut &P, int level) {
   for (auto &k : P.chunks) m.chunks.push_back({k.t0, k.nt});
 }
 
+bool use_group_v1();
+
+// The min-hash kernels also write each key's top byte (the coarse bin) for
+// the byte histogram: single rank, stable grouping, rows in generator order.
+bool use_kbin(const sg_graph *g, const PassOut &P) {
+  return !g->xch && use_group_v1() && P.perm.p == nullptr && !getenv("SG_NO_KBIN");
+}
+
 void plan_pass_uncached(sg_graph *g, PassOut &P) {
   const int64_t nr = P.nrows, c = P.c;
-  const double keys_t = 8.0 * (double)P.key_stride;             // keys of one trial
+  // keys of one trial (+ their top bytes; unplanned, they over-committed the
+  // eager plans of the c = 400 sweep points)
+  const double keys_t = (use_kbin(g, P) ? 9.0 : 8.0) * (double)P.key_stride;
   const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;   // scratch per trial
   const double members = 4.125 * (double)nr * (double)c + (1 << 20);
   // headroom: the plan's buffers are carved from one stream-ordered pool, and
@@ -440,7 +450,7 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_s
   dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
   // top key bytes for the coarse histogram (1 B instead of 8 B per pair):
   // single rank, stable grouping, rows in generator order
-  const bool want_kbin = !g->xch && use_group_v1() && P.perm.p == nullptr && !getenv("SG_NO_KBIN");
+  const bool want_kbin = use_kbin(g, P);
   if (want_kbin) dalloc(g, ch.kbin, (size_t)ch.nt * (size_t)P.key_stride);
   DBuf &ctr = ch.ctr;
   dalloc(g, ctr, 16);
