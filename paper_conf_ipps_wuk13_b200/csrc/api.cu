@@ -330,6 +330,7 @@ void plan_pass(sg_graph *g, PassOut &P, int level) {
   if (!g->xch && m.nrows == P.nrows && m.c == P.c && m.live == g->bytes_live &&
       m.cached == g->bytes_cached) {
     P.deferred = m.deferred;
+    P.kbin = m.kbin;
     P.chunks.clear();
     for (auto &tc : m.chunks) {
       KeyChunk k;
@@ -345,23 +346,23 @@ void plan_pass(sg_graph *g, PassOut &P, int level) {
   m.nrows = P.nrows;
   m.c = P.c;
   m.deferred = P.deferred;
+  m.kbin = P.kbin;
   m.chunks.clear();
   for (auto &k : P.chunks) m.chunks.push_back({k.t0, k.nt});
 }
 
 bool use_group_v1();
 
-// The min-hash kernels also write each key's top byte (the coarse bin) for
-// the byte histogram: single rank, stable grouping, rows in generator order.
-bool use_kbin(const sg_graph *g, const PassOut &P) {
+// The min-hash kernels may also write each key's top byte (the coarse bin)
+// for the byte histogram: single rank, stable grouping, rows in generator
+// order, and only when the plan leaves room for them (below).
+bool kbin_eligible(const sg_graph *g, const PassOut &P) {
   return !g->xch && use_group_v1() && P.perm.p == nullptr && !getenv("SG_NO_KBIN");
 }
 
 void plan_pass_uncached(sg_graph *g, PassOut &P) {
   const int64_t nr = P.nrows, c = P.c;
-  // keys of one trial (+ their top bytes; unplanned, they over-committed the
-  // eager plans of the c = 400 sweep points)
-  const double keys_t = (use_kbin(g, P) ? 9.0 : 8.0) * (double)P.key_stride;
+  const double keys_t = 8.0 * (double)P.key_stride;             // keys of one trial
   const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;   // scratch per trial
   const double members = 4.125 * (double)nr * (double)c + (1 << 20);
   // headroom: the plan's buffers are carved from one stream-ordered pool, and
@@ -369,8 +370,9 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
   // allocations then fail, the pool is trimmed and re-mapped inside the timed
   // stages: measured 0.26-1.6 s group2 swings on hub2m); plan against 90 %
   // of the available bytes minus 4 GB
-  const double avail = g->mem_budget > 0 ? (double)avail_bytes(g)        // test hook: exact budget
-                                         : 0.9 * (double)avail_bytes(g) - 4.0e9;
+  const double raw = (double)avail_bytes(g);
+  const double avail = g->mem_budget > 0 ? raw        // test hook: exact budget
+                                         : 0.9 * raw - 4.0e9;
   int64_t ct = (int64_t)((avail - members - keys_t * c) / scr_t);
   P.deferred = false;
   if (g->xch) {
@@ -404,6 +406,18 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
     k.t0 = (int32_t)t;
     k.nt = (int32_t)std::min<int64_t>(per, c - t);
     P.chunks.push_back(k);
+  }
+  // the key bytes (1 B per resident key) ride in the plan's headroom when it
+  // has room for them; otherwise the histogram reads the keys (unplanned,
+  // they over-committed the eager plan of the s = 3, c = 400 sweep point:
+  // group2 581 -> 1455 ms; planned at 9 B per key they split gos2m into 7
+  // trial chunks instead of 4: +8 ms)
+  P.kbin = false;
+  if (kbin_eligible(g, P)) {
+    const double resident_keys = P.deferred ? (double)per : (double)c;
+    const double need = members + resident_keys * keys_t + (double)per * scr_t +
+                        resident_keys * (double)P.key_stride;
+    P.kbin = need <= (g->mem_budget > 0 ? raw : 0.97 * raw);
   }
 }
 
@@ -450,7 +464,7 @@ void compute_chunk(sg_graph *g, PassOut &P, KeyChunk &ch, int st_hash, bool on_s
   dalloc(g, ch.keys, (size_t)ch.nt * (size_t)P.key_stride * 8);
   // top key bytes for the coarse histogram (1 B instead of 8 B per pair):
   // single rank, stable grouping, rows in generator order
-  const bool want_kbin = use_kbin(g, P);
+  const bool want_kbin = P.kbin;
   if (want_kbin) dalloc(g, ch.kbin, (size_t)ch.nt * (size_t)P.key_stride);
   DBuf &ctr = ch.ctr;
   dalloc(g, ctr, 16);

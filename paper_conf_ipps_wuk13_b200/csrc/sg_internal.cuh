@@ -100,6 +100,7 @@ struct PassOut {
   const uint32_t *entries = nullptr;  // row entries (pass I: col; pass II: G_I members)
   std::vector<KeyChunk> chunks; // trial chunks sized to the free HBM
   bool deferred = false;        // keys computed chunk by chunk inside group_by_shingle
+  bool kbin = false;            // the min-hash kernels also write the keys' top bytes
   std::vector<int64_t> blocks;  // row blocks in generator order (multi-rank exchange pieces)
   // pass II, one rank: key positions in length-class order;
   // key position i belongs to row perm[i]; positions [0, n_split) are rows of
@@ -191,7 +192,7 @@ struct sg_graph {
   // the same allocation state
   struct PlanMemo {
     int64_t nrows = -1, c = -1, live = -1, cached = -1;
-    bool deferred = false;
+    bool deferred = false, kbin = false;
     std::vector<std::pair<int32_t, int32_t>> chunks;
   } plan_memo[2];
   std::vector<sg::DBuf> cache;  // freed blocks kept for reuse (best fit)
