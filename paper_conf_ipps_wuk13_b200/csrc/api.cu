@@ -360,21 +360,20 @@ bool kbin_eligible(const sg_graph *g, const PassOut &P) {
   return !g->xch && use_group_v1() && P.perm.p == nullptr && !getenv("SG_NO_KBIN");
 }
 
-void plan_pass_uncached(sg_graph *g, PassOut &P) {
+// One plan for `kb` bytes per resident key: eager (all keys resident, the
+// scratch of `per` trials beside them) or deferred (keys of one chunk).
+struct Plan {
+  bool deferred = false;
+  int64_t per = 0, nch = 0;
+};
+
+Plan make_plan(sg_graph *g, const PassOut &P, double kb, double avail) {
   const int64_t nr = P.nrows, c = P.c;
-  const double keys_t = 8.0 * (double)P.key_stride;             // keys of one trial
+  const double keys_t = kb * (double)P.key_stride;              // keys of one trial
   const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;   // scratch per trial
   const double members = 4.125 * (double)nr * (double)c + (1 << 20);
-  // headroom: the plan's buffers are carved from one stream-ordered pool, and
-  // a plan that fills the device to the last gigabyte fragments it (the
-  // allocations then fail, the pool is trimmed and re-mapped inside the timed
-  // stages: measured 0.26-1.6 s group2 swings on hub2m); plan against 90 %
-  // of the available bytes minus 4 GB
-  const double raw = (double)avail_bytes(g);
-  const double avail = g->mem_budget > 0 ? raw        // test hook: exact budget
-                                         : 0.9 * raw - 4.0e9;
+  Plan pl;
   int64_t ct = (int64_t)((avail - members - keys_t * c) / scr_t);
-  P.deferred = false;
   if (g->xch) {
     // multi-rank: all keys are kept until their exchange (eager), sorted keys
     // are kept for the getters, send + receive buffers per chunk; every rank
@@ -385,7 +384,7 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
     if (ct < 1) fail(g, SG_ENOMEM, "multi-rank pass needs all keys resident; not enough HBM");
   } else if (ct < 1) {
     ct = (int64_t)((avail - members) / (keys_t + scr_t));
-    P.deferred = true;
+    pl.deferred = true;
     if (ct < 1) {
       char buf[160];
       snprintf(buf, sizeof buf, "pass needs more HBM than available (%.0f B for the members alone)",
@@ -394,30 +393,56 @@ void plan_pass_uncached(sg_graph *g, PassOut &P) {
     }
   }
   ct = std::min<int64_t>(ct, c);
-  const int64_t nch = (c + ct - 1) / ct;
-  int64_t per = (c + nch - 1) / nch;
+  pl.nch = (c + ct - 1) / ct;
+  pl.per = (c + pl.nch - 1) / pl.nch;
   // whole 32-trial groups per chunk: the min-hash runs 32 trials per lane
   // pass and a tail pass (c mod 32 trials) costs a full pass per row, so
   // e.g. 200 = 64+64+64+8 (7 passes) rather than 67+67+66 (11 passes)
-  if (per < c && per >= 32) per = per / 32 * 32;
-  P.chunks.clear();
-  for (int64_t t = 0; t < c; t += per) {
-    KeyChunk k;
-    k.t0 = (int32_t)t;
-    k.nt = (int32_t)std::min<int64_t>(per, c - t);
-    P.chunks.push_back(k);
-  }
-  // the key bytes (1 B per resident key) ride in the plan's headroom when it
-  // has room for them; otherwise the histogram reads the keys (unplanned,
-  // they over-committed the eager plan of the s = 3, c = 400 sweep point:
-  // group2 581 -> 1455 ms; planned at 9 B per key they split gos2m into 7
-  // trial chunks instead of 4: +8 ms)
+  if (pl.per < c && pl.per >= 32) pl.per = pl.per / 32 * 32;
+  pl.nch = (c + pl.per - 1) / pl.per;
+  return pl;
+}
+
+void plan_pass_uncached(sg_graph *g, PassOut &P) {
+  const int64_t nr = P.nrows, c = P.c;
+  // headroom: the plan's buffers are carved from one stream-ordered pool, and
+  // a plan that fills the device to the last gigabyte fragments it (the
+  // allocations then fail, the pool is trimmed and re-mapped inside the timed
+  // stages: measured 0.26-1.6 s group2 swings on hub2m); plan against 90 %
+  // of the available bytes minus 4 GB
+  const double raw = (double)avail_bytes(g);
+  const double avail = g->mem_budget > 0 ? raw        // test hook: exact budget
+                                         : 0.9 * raw - 4.0e9;
+  Plan pl = make_plan(g, P, 8.0, avail);
   P.kbin = false;
   if (kbin_eligible(g, P)) {
-    const double resident_keys = P.deferred ? (double)per : (double)c;
-    const double need = members + resident_keys * keys_t + (double)per * scr_t +
-                        resident_keys * (double)P.key_stride;
-    P.kbin = need <= (g->mem_budget > 0 ? raw : 0.97 * raw);
+    // The key bytes of the byte histogram (1 B per resident key): planned at
+    // 9 B per key when that plan has no more chunks than the 8 B one; else
+    // carried in the 8 B plan's headroom when the device still holds them;
+    // else left out (measured: unplanned they over-committed the eager plan
+    // of the s = 3, c = 400 sweep point, 2.7 s per step; planned, its
+    // deferred 5-chunk plan runs in 0.64 s; planned at 9 B they split gos2m
+    // into 7 trial chunks instead of 4, +8 ms, while the 4-chunk plan holds
+    // them in its headroom)
+    const Plan p9 = make_plan(g, P, 9.0, avail);
+    if (p9.nch <= pl.nch) {
+      pl = p9;
+      P.kbin = true;
+    } else {
+      const double scr_t = scratch_per_pair(nr) * (double)nr + 65536.0 * 8;
+      const double members = 4.125 * (double)nr * (double)c + (1 << 20);
+      const double resident = pl.deferred ? (double)pl.per : (double)c;
+      const double need = members + resident * 9.0 * (double)P.key_stride + (double)pl.per * scr_t;
+      P.kbin = need <= (g->mem_budget > 0 ? raw : 0.97 * raw);
+    }
+  }
+  P.deferred = pl.deferred;
+  P.chunks.clear();
+  for (int64_t t = 0; t < c; t += pl.per) {
+    KeyChunk k;
+    k.t0 = (int32_t)t;
+    k.nt = (int32_t)std::min<int64_t>(pl.per, c - t);
+    P.chunks.push_back(k);
   }
 }
 
